@@ -1,0 +1,237 @@
+// cellfn.cuh -- the compiled-in cell functions f of the LDDP-Plus recurrence
+//     table[i][j] = f(L, UL, U, UR)          [L30 §I], [L94 §II], RS(i,j) [L90]
+// and the initialisation each f implies [L300-L313].  Every functor declares its contributing
+// set (kMask, Table I [L124-L142]) and supplies:
+//   top(gc)   value of the row above the f-region (table row 0) at global column gc in [-1, n]
+//   left(i)   value of the column left of the f-region at row i   (table column 0)
+//   right(i)  value right of the last column (only read through UR)
+//   row_ctx / col_ctx / load   per-row, per-column and per-cell inputs
+//   f(...)    the cell update; writes the table-output element into `o`
+// Readings of the paper (R1..R9) are listed in DESIGN.md §3.
+#pragma once
+#include <cstdint>
+#include <climits>
+#include "params.h"
+
+namespace lddp {
+
+enum : uint32_t { NB_L = 1u, NB_UL = 2u, NB_U = 4u, NB_UR = 8u };
+enum ScoreKind { SCORE_NONE = 0, SCORE_LAST_CELL = 1, SCORE_ROW_MIN = 2 };
+
+// ---------------------------------------------------------------------------------------- LCS
+// [L88] Fig. 1(c) contributing set {L,UL,U}; textbook recurrence (reading R1) in the exact
+// integer form max(U, L, UL + [a_i = b_j]) (equal to the textbook branch form because
+// adjacent LCS cells differ by at most 1).
+struct CellLCS {
+  using T = int32_t;
+  using RowCtx = int32_t;
+  using ColCtx = int32_t;
+  using GridT = int32_t;
+  using OutT = int32_t;
+  static constexpr uint32_t kMask = NB_L | NB_UL | NB_U;
+  static constexpr bool kGridIn = false;
+  static constexpr int kScore = SCORE_LAST_CELL;
+  __device__ static RowCtx row_ctx(const FillParams& p, int64_t i) {
+    return static_cast<const uint8_t*>(p.a)[i];
+  }
+  __device__ static ColCtx col_ctx(const FillParams& p, int gc) {
+    return static_cast<const uint8_t*>(p.b)[gc];
+  }
+  __device__ static T top(const FillParams&, int) { return 0; }
+  __device__ static T left(const FillParams&, int64_t) { return 0; }
+  __device__ static T right(const FillParams&, int64_t) { return 0; }
+  __device__ static GridT load(const FillParams&, int64_t, int) { return 0; }
+  __device__ __forceinline__ static T f(T L, T UL, T U, T, RowCtx a, ColCtx b, GridT, int64_t,
+                                        int, int, OutT& o) {
+    T v = max(max(U, L), UL + (a == b ? 1 : 0));
+    o = v;
+    return v;
+  }
+};
+
+// -------------------------------------------------------------------------------- Levenshtein
+// [L319-L329] §VI.A with the restored min (reading R7): boundary max(i,j); equal characters
+// copy UL, else 1 + min(U, L, UL).
+struct CellLev {
+  using T = int32_t;
+  using RowCtx = int32_t;
+  using ColCtx = int32_t;
+  using GridT = int32_t;
+  using OutT = int32_t;
+  static constexpr uint32_t kMask = NB_L | NB_UL | NB_U;
+  static constexpr bool kGridIn = false;
+  static constexpr int kScore = SCORE_LAST_CELL;
+  __device__ static RowCtx row_ctx(const FillParams& p, int64_t i) {
+    return static_cast<const uint8_t*>(p.a)[i];
+  }
+  __device__ static ColCtx col_ctx(const FillParams& p, int gc) {
+    return static_cast<const uint8_t*>(p.b)[gc];
+  }
+  __device__ static T top(const FillParams&, int gc) { return gc + 1; }           // f(0, gc+1)
+  __device__ static T left(const FillParams&, int64_t i) { return (T)(i + 1); }   // f(i+1, 0)
+  __device__ static T right(const FillParams&, int64_t) { return 0; }
+  __device__ static GridT load(const FillParams&, int64_t, int) { return 0; }
+  __device__ __forceinline__ static T f(T L, T UL, T U, T, RowCtx a, ColCtx b, GridT, int64_t,
+                                        int, int, OutT& o) {
+    T v = (a == b) ? UL : 1 + min(min(U, L), UL);
+    o = v;
+    return v;
+  }
+};
+
+// ---------------------------------------------------------------------------------------- DTW
+// [L26] + reading R2: D[0][0] = 0, D[i][0] = D[0][j] = +inf; binary32
+// D = |x_i - y_j| + min(min(U, L), UL) -- the oracle's exact operation sequence (one rounded
+// subtraction, exact mins, one rounded add), so the result is bit-identical.
+struct CellDTW {
+  using T = float;
+  using RowCtx = float;
+  using ColCtx = float;
+  using GridT = float;
+  using OutT = float;
+  static constexpr uint32_t kMask = NB_L | NB_UL | NB_U;
+  static constexpr bool kGridIn = false;
+  static constexpr int kScore = SCORE_LAST_CELL;
+  __device__ static RowCtx row_ctx(const FillParams& p, int64_t i) {
+    return static_cast<const float*>(p.a)[i];
+  }
+  __device__ static ColCtx col_ctx(const FillParams& p, int gc) {
+    return static_cast<const float*>(p.b)[gc];
+  }
+  __device__ static T top(const FillParams&, int gc) { return gc == -1 ? 0.0f : __int_as_float(0x7f800000); }
+  __device__ static T left(const FillParams&, int64_t) { return __int_as_float(0x7f800000); }
+  __device__ static T right(const FillParams&, int64_t) { return __int_as_float(0x7f800000); }
+  __device__ static GridT load(const FillParams&, int64_t, int) { return 0.0f; }
+  __device__ __forceinline__ static T f(T L, T UL, T U, T, RowCtx x, ColCtx y, GridT, int64_t,
+                                        int, int, OutT& o) {
+    float cost = fabsf(__fsub_rn(x, y));
+    float v = __fadd_rn(cost, fminf(fminf(U, L), UL));
+    o = v;
+    return v;
+  }
+};
+
+// ------------------------------------------------------------------------- Floyd-Steinberg
+// [L341-L344] §VI.B.  The carried cell value is the diffusion error e of the pixel.  Pull form
+// of the raster push form: the four contributions reach pixel (i,j) in raster order UL, U, UR,
+// L, so v = (((in + e_UL*1/16) + e_U*5/16) + e_UR*3/16) + e_L*7/16 with every product and sum
+// rounded separately (__fmul_rn / __fadd_rn are never contracted to FFMA) -- bit-identical to
+// the oracle.  Absent neighbours carry e = 0 (+0.0 adds are exact).  Threshold 128, ties to
+// 255 (reading R3); e = v - out (reading R4).
+struct CellFS {
+  using T = float;
+  using RowCtx = int32_t;
+  using ColCtx = int32_t;
+  using GridT = float;
+  using OutT = uint8_t;
+  static constexpr uint32_t kMask = NB_L | NB_UL | NB_U | NB_UR;
+  static constexpr bool kGridIn = true;
+  static constexpr int kScore = SCORE_NONE;
+  __device__ static RowCtx row_ctx(const FillParams&, int64_t) { return 0; }
+  __device__ static ColCtx col_ctx(const FillParams&, int) { return 0; }
+  __device__ static T top(const FillParams&, int) { return 0.0f; }
+  __device__ static T left(const FillParams&, int64_t) { return 0.0f; }
+  __device__ static T right(const FillParams&, int64_t) { return 0.0f; }
+  __device__ static GridT load(const FillParams& p, int64_t i, int c) {
+    return (float)__ldg(static_cast<const uint8_t*>(p.grid) + i * p.grid_pitch + c);
+  }
+  __device__ __forceinline__ static T f(T L, T UL, T U, T UR, RowCtx, ColCtx, GridT in, int64_t,
+                                        int, int, OutT& o) {
+    float v = __fadd_rn(in, __fmul_rn(UL, 0.0625f));
+    v = __fadd_rn(v, __fmul_rn(U, 0.3125f));
+    v = __fadd_rn(v, __fmul_rn(UR, 0.1875f));
+    v = __fadd_rn(v, __fmul_rn(L, 0.4375f));
+    const bool hi = v >= 128.0f;
+    o = hi ? (uint8_t)255 : (uint8_t)0;
+    return hi ? __fsub_rn(v, 255.0f) : v;
+  }
+};
+
+// ------------------------------------------------------------------------------ MIN_PATH3
+// [L350-L367] §VI.C checkerboard, reading R6: f[0][j] = c[0][j]; f = c + min over the in-range
+// {UL, U, UR}.  Out-of-range neighbours are INT_MAX, used only as min operands.  The row above
+// row 0 is 0 inside the grid, so f[0][j] = c[0][j] + 0.
+struct CellMinPath3 {
+  using T = int32_t;
+  using RowCtx = int32_t;
+  using ColCtx = int32_t;
+  using GridT = int32_t;
+  using OutT = int32_t;
+  static constexpr uint32_t kMask = NB_UL | NB_U | NB_UR;
+  static constexpr bool kGridIn = true;
+  static constexpr int kScore = SCORE_ROW_MIN;
+  __device__ static RowCtx row_ctx(const FillParams&, int64_t) { return 0; }
+  __device__ static ColCtx col_ctx(const FillParams&, int) { return 0; }
+  __device__ static T top(const FillParams& p, int gc) {
+    return (gc >= 0 && gc < p.cols_total) ? 0 : INT_MAX;
+  }
+  __device__ static T left(const FillParams&, int64_t) { return INT_MAX; }
+  __device__ static T right(const FillParams&, int64_t) { return INT_MAX; }
+  __device__ static GridT load(const FillParams& p, int64_t i, int c) {
+    return __ldg(static_cast<const int32_t*>(p.grid) + i * p.grid_pitch + c);
+  }
+  __device__ __forceinline__ static T f(T, T UL, T U, T UR, RowCtx, ColCtx, GridT g, int64_t,
+                                        int, int, OutT& o) {
+    T v = g + min(min(UL, U), UR);
+    o = v;
+    return v;
+  }
+};
+
+// ------------------------------------------------------------------------------ MIN2_PLUS
+// [L298] §V.B Horizontal case-1 synthetic f = min(UL, U) + c; row 0 = init (reading R8);
+// UL at j = 0 is INT_MAX (excluded).
+struct CellMin2Plus {
+  using T = int32_t;
+  using RowCtx = int32_t;
+  using ColCtx = int32_t;
+  using GridT = int32_t;
+  using OutT = int32_t;
+  static constexpr uint32_t kMask = NB_UL | NB_U;
+  static constexpr bool kGridIn = true;
+  static constexpr int kScore = SCORE_ROW_MIN;
+  __device__ static RowCtx row_ctx(const FillParams&, int64_t) { return 0; }
+  __device__ static ColCtx col_ctx(const FillParams&, int) { return 0; }
+  __device__ static T top(const FillParams&, int) { return 0; }
+  __device__ static T left(const FillParams&, int64_t) { return INT_MAX; }
+  __device__ static T right(const FillParams&, int64_t) { return INT_MAX; }
+  __device__ static GridT load(const FillParams& p, int64_t i, int c) {
+    return __ldg(static_cast<const int32_t*>(p.grid) + i * p.grid_pitch + c);
+  }
+  __device__ __forceinline__ static T f(T, T UL, T U, T, RowCtx, ColCtx, GridT g, int64_t i,
+                                        int, int pc, OutT& o) {
+    T v = (i == 0) ? g : min(UL, U) + pc;
+    o = v;
+    return v;
+  }
+};
+
+// --------------------------------------------------------------------------- DIAG_MAXPLUS
+// [L298] §V.B Inverted-L synthetic f = max(cell_{i,j}, f(i-1,j-1)) + c, cell = init (reading
+// R9); row 0 and column 0 are init.
+struct CellDiagMaxPlus {
+  using T = int32_t;
+  using RowCtx = int32_t;
+  using ColCtx = int32_t;
+  using GridT = int32_t;
+  using OutT = int32_t;
+  static constexpr uint32_t kMask = NB_UL;
+  static constexpr bool kGridIn = true;
+  static constexpr int kScore = SCORE_NONE;
+  __device__ static RowCtx row_ctx(const FillParams&, int64_t) { return 0; }
+  __device__ static ColCtx col_ctx(const FillParams&, int) { return 0; }
+  __device__ static T top(const FillParams&, int) { return 0; }
+  __device__ static T left(const FillParams&, int64_t) { return 0; }
+  __device__ static T right(const FillParams&, int64_t) { return 0; }
+  __device__ static GridT load(const FillParams& p, int64_t i, int c) {
+    return __ldg(static_cast<const int32_t*>(p.grid) + i * p.grid_pitch + c);
+  }
+  __device__ __forceinline__ static T f(T, T UL, T, T, RowCtx, ColCtx, GridT g, int64_t i,
+                                        int gc, int pc, OutT& o) {
+    T v = (i == 0 || gc == 0) ? g : max(g, UL) + pc;
+    o = v;
+    return v;
+  }
+};
+
+}  // namespace lddp

@@ -1,0 +1,83 @@
+// invl.cu -- Inverted-L category kernel ("the remaining pattern", t = min(i,j)) [L197-L215],
+// Fig. 2(c), contributing set {UL} (Table I [L129], [L203]).
+//
+// With UL as the only dependency, every diagonal d = j - i is an independent chain.  The paper
+// processes shrinking inverted-L shells with one launch each [L205] and notes the horizontal
+// case-1 schedule is better for coalescing [L215], [L296-L298].  On B200 the natural form is
+// neither: one lane per diagonal chain, 32 adjacent diagonals per warp, walking rows in
+// lockstep -- so lane l touches column i + d0 + l of row i: every row step is one coalesced
+// 128-byte load (and store), no inter-thread dependency at all, pure HBM streaming with an
+// unrolled prefetch of UNR rows per lane.
+#include <cstdint>
+#include "cellfn.cuh"
+#include "params.h"
+#include "sync.cuh"
+
+namespace lddp {
+
+constexpr int kInvlWarps = 8;
+constexpr int kInvlUnroll = 8;
+
+template <class F, bool TABLE>
+__global__ void __launch_bounds__(kInvlWarps * 32) invl_kernel(const FillParams p) {
+  using T = typename F::T;
+  using G = typename F::GridT;
+  static_assert(F::kMask == NB_UL, "inverted-L category: contributing set must be {UL}");
+  const int lane = threadIdx.x & 31;
+  const int64_t H = p.rows;
+  const int W = p.cols;
+  const int64_t nd = H + W - 1;                      // diagonals d = j - i in [-(H-1), W-1]
+  const int64_t nwarps_total = (nd + 31) / 32;
+  const int64_t gw0 = (int64_t)blockIdx.x * kInvlWarps + (threadIdx.x >> 5);
+  const int64_t gstride = (int64_t)gridDim.x * kInvlWarps;
+  for (int64_t gw = gw0; gw < nwarps_total; gw += gstride) {
+    const int64_t d = -(H - 1) + gw * 32 + lane;     // this lane's diagonal
+    const bool live = d <= (int64_t)W - 1;
+    // rows this warp visits: union of its lanes' chains
+    const int64_t dlo = -(H - 1) + gw * 32;
+    const int64_t dhi = min((int64_t)W - 1, dlo + 31);
+    const int64_t ibeg = max((int64_t)0, -dhi);
+    const int64_t iend = min(H, (int64_t)W - dlo);   // exclusive
+    T v = T(0);
+    for (int64_t i0 = ibeg; i0 < iend; i0 += kInvlUnroll) {
+      G g[kInvlUnroll];
+#pragma unroll
+      for (int u = 0; u < kInvlUnroll; ++u) {
+        const int64_t i = i0 + u;
+        const int64_t j = i + d;
+        g[u] = (live && i < iend && j >= 0 && j < W) ? F::load(p, i, (int)j) : G(0);
+      }
+#pragma unroll
+      for (int u = 0; u < kInvlUnroll; ++u) {
+        const int64_t i = i0 + u;
+        const int64_t j = i + d;
+        if (live && i < iend && j >= 0 && j < W) {
+          typename F::OutT o;
+          v = F::f(v, v, v, v, typename F::RowCtx(0), typename F::ColCtx(0), g[u], i,
+                   (int)j + p.col0, p.param_c, o);
+          if (TABLE) static_cast<typename F::OutT*>(p.table)[i * p.table_pitch + j] = o;
+          if (i == H - 1 && p.last_row != nullptr) static_cast<T*>(p.last_row)[j] = v;
+          if (j == W - 1 && p.last_col != nullptr) static_cast<T*>(p.last_col)[i] = v;
+        }
+      }
+    }
+  }
+}
+
+template <class F>
+static cudaError_t launch_il(const FillParams& p, int grid, cudaStream_t s) {
+  if (p.table != nullptr)
+    invl_kernel<F, true><<<grid, kInvlWarps * 32, 0, s>>>(p);
+  else
+    invl_kernel<F, false><<<grid, kInvlWarps * 32, 0, s>>>(p);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_invl(int func, const FillParams& p, int grid, cudaStream_t s) {
+  switch (func) {
+    case 4: return launch_il<CellDiagMaxPlus>(p, grid, s);
+    default: return cudaErrorInvalidValue;
+  }
+}
+
+}  // namespace lddp

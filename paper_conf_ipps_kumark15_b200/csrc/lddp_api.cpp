@@ -1,0 +1,752 @@
+// lddp_api.cpp -- C ABI of liblddp.so (include/lddp.h): classification (Table I), planning,
+// workspace layout, fills (single GPU, host-buffer, multi-GPU column strips) and status.
+//
+// The planner is the paper's "framework maps the function to a pattern" step [L113]: the
+// contributing set of the compiled-in f is checked against the requested category's schedule
+// (Fig. 2 [L117-L122]); the launch geometry replaces the paper's empirical t_switch / t_share
+// tuning [L288-L294] (there is no CPU share on B200: the fill is GPU-only).
+#include "../../include/lddp.h"
+
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <atomic>
+#include <cstdarg>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <mutex>
+#include <new>
+#include <string>
+
+#include "params.h"
+#include "sync.cuh"
+
+namespace lddp {
+int wf_dispatch_lcs(int, int, bool, const FillParams*, int, cudaStream_t);
+int wf_dispatch_lev(int, int, bool, const FillParams*, int, cudaStream_t);
+int wf_dispatch_dtw(int, int, bool, const FillParams*, int, cudaStream_t);
+int wf_dispatch_fs(int, int, bool, const FillParams*, int, cudaStream_t);
+int wf_dispatch_minpath3(int, int, bool, const FillParams*, int, cudaStream_t);
+int wf_dispatch_min2plus(int, int, bool, const FillParams*, int, cudaStream_t);
+int wf_dispatch_diagmaxplus(int, int, bool, const FillParams*, int, cudaStream_t);
+}  // namespace lddp
+
+using lddp::FillParams;
+
+namespace {
+
+thread_local std::string g_last_error;
+std::atomic<uint64_t> g_epoch{1};
+
+lddp_status fail(lddp_status s, const char* fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof buf, fmt, ap);
+  va_end(ap);
+  g_last_error = buf;
+  return s;
+}
+
+lddp_status cuda_fail(cudaError_t e, const char* what) {
+  return fail(LDDP_ERR_CUDA, "%s: %s (%s)", what, cudaGetErrorName(e), cudaGetErrorString(e));
+}
+
+#define CUDA_TRY(expr)                                              \
+  do {                                                              \
+    cudaError_t _e = (expr);                                        \
+    if (_e != cudaSuccess) return cuda_fail(_e, #expr);             \
+  } while (0)
+
+// --------------------------------------------------------------------- Table I / Fig. 2
+// Table I [L124-L142]: pattern of every non-empty contributing set (bits L=1, UL=2, U=4, UR=8).
+const int kTable1[16] = {
+    -1,                     // {} (not a valid f)
+    LDDP_PAT_VERTICAL,      // {L}              [L133]
+    LDDP_PAT_INVERTED_L,    // {UL}             [L129]
+    LDDP_PAT_VERTICAL,      // {L,UL}           [L137]
+    LDDP_PAT_HORIZONTAL,    // {U}              [L127]
+    LDDP_PAT_ANTI_DIAGONAL, // {L,U}            [L135]
+    LDDP_PAT_HORIZONTAL,    // {UL,U}           [L131]
+    LDDP_PAT_ANTI_DIAGONAL, // {L,UL,U}         [L139]
+    LDDP_PAT_MINVERTED_L,   // {UR}             [L126]
+    LDDP_PAT_KNIGHT_MOVE,   // {L,UR}           [L134]
+    LDDP_PAT_HORIZONTAL,    // {UL,UR}          [L130]
+    LDDP_PAT_KNIGHT_MOVE,   // {L,UL,UR}        [L138]
+    LDDP_PAT_HORIZONTAL,    // {U,UR}           [L128]
+    LDDP_PAT_KNIGHT_MOVE,   // {L,U,UR}         [L136]
+    LDDP_PAT_HORIZONTAL,    // {UL,U,UR}        [L132]
+    LDDP_PAT_KNIGHT_MOVE,   // {L,UL,U,UR}      [L140]
+};
+
+// Dependencies each category's schedule strictly orders (Fig. 2 [L117-L122], 0-based t):
+//   prev-row t=i: UL, U, UR (t-1); anti-diagonal t=i+j: L (t-1), UL (t-2), U (t-1);
+//   knight-move t=2i+j: L (t-1), UL (t-3), U (t-2), UR (t-1); inverted-L t=min(i,j): UL only.
+uint32_t category_allows(int cat) {
+  switch (cat) {
+    case LDDP_CAT_PREV_ROW: return LDDP_NB_UL | LDDP_NB_U | LDDP_NB_UR;
+    case LDDP_CAT_ANTI_DIAGONAL: return LDDP_NB_L | LDDP_NB_UL | LDDP_NB_U;
+    case LDDP_CAT_KNIGHT_MOVE: return LDDP_NB_L | LDDP_NB_UL | LDDP_NB_U | LDDP_NB_UR;
+    case LDDP_CAT_INVERTED_L: return LDDP_NB_UL;
+    default: return 0;
+  }
+}
+
+uint32_t func_mask(int f) {
+  switch (f) {
+    case LDDP_F_LCS: return LDDP_NB_L | LDDP_NB_UL | LDDP_NB_U;
+    case LDDP_F_DTW: return LDDP_NB_L | LDDP_NB_UL | LDDP_NB_U;
+    case LDDP_F_FS_DITHER: return LDDP_NB_L | LDDP_NB_UL | LDDP_NB_U | LDDP_NB_UR;
+    case LDDP_F_MIN_PATH3: return LDDP_NB_UL | LDDP_NB_U | LDDP_NB_UR;
+    case LDDP_F_DIAG_MAXPLUS: return LDDP_NB_UL;
+    case LDDP_F_MIN2_PLUS: return LDDP_NB_UL | LDDP_NB_U;
+    case LDDP_F_LEVENSHTEIN: return LDDP_NB_L | LDDP_NB_UL | LDDP_NB_U;
+    default: return 0;
+  }
+}
+
+bool seq_func(int f) { return f == LDDP_F_LCS || f == LDDP_F_DTW || f == LDDP_F_LEVENSHTEIN; }
+size_t cell_bytes(int) { return 4; }   // int32 or binary32 cells for every f
+size_t seq_elt_bytes(int f) { return f == LDDP_F_DTW ? 4 : 1; }
+size_t grid_elt_bytes(int f) { return f == LDDP_F_FS_DITHER ? 1 : 4; }
+size_t table_elt_bytes(int f) { return f == LDDP_F_FS_DITHER ? 1 : 4; }
+
+int wf_dispatch(int func, int op, int variant, bool table, const FillParams* p, int grid,
+                cudaStream_t s) {
+  switch (func) {
+    case LDDP_F_LCS: return lddp::wf_dispatch_lcs(op, variant, table, p, grid, s);
+    case LDDP_F_LEVENSHTEIN: return lddp::wf_dispatch_lev(op, variant, table, p, grid, s);
+    case LDDP_F_DTW: return lddp::wf_dispatch_dtw(op, variant, table, p, grid, s);
+    case LDDP_F_FS_DITHER: return lddp::wf_dispatch_fs(op, variant, table, p, grid, s);
+    case LDDP_F_MIN_PATH3: return lddp::wf_dispatch_minpath3(op, variant, table, p, grid, s);
+    case LDDP_F_MIN2_PLUS: return lddp::wf_dispatch_min2plus(op, variant, table, p, grid, s);
+    case LDDP_F_DIAG_MAXPLUS: return lddp::wf_dispatch_diagmaxplus(op, variant, table, p, grid, s);
+    default: return -1;
+  }
+}
+
+// variant geometry: rows per lane R, intra-lane skew SIG, extra lag E
+struct VariantGeom { int id, R, SIG, E; };
+const VariantGeom kVariants[] = {
+    {0, 4, 0, 2}, {1, 4, 1, 1}, {2, 2, 1, 1}, {3, 8, 1, 1}, {10, 1, 2, 2}, {11, 2, 2, 2},
+};
+const VariantGeom* variant_geom(int id) {
+  for (const auto& v : kVariants)
+    if (v.id == id) return &v;
+  return nullptr;
+}
+constexpr int kWfWarps = 4;           // must match wavefront_launch.cuh
+constexpr int kPrevBandRows = 32;     // must match prevrow.cu
+constexpr int kPrevBW = 128;
+constexpr int kPrevRing = 4;
+constexpr int kPrevThreads = 256;
+constexpr int kInvlThreads = 256;
+
+int env_int(const char* name, int dflt) {
+  const char* v = getenv(name);
+  return (v && *v) ? atoi(v) : dflt;
+}
+
+}  // namespace
+
+// ------------------------------------------------------------------------------ plan object
+struct lddp_plan_s {
+  lddp_desc desc;
+  int kind;          // 0 = wavefront (anti-diag / knight), 1 = prev-row, 2 = inverted-L
+  int variant;       // wavefront variant id
+  int R, SIG, E;
+  int sms;
+  int grid;
+  int occupancy;
+  // wavefront geometry
+  int64_t strip_rows;
+  int nstrips;
+  int nchunks;
+  int64_t row0;
+  int64_t bnd_stride;
+  // prev-row geometry
+  int nblocks;
+  int nbands;
+  // workspace layout (bytes)
+  size_t off_prog, off_bnd, ws_bytes;
+  // own workspace + host-fill staging
+  void* own_ws;
+  std::mutex mu;
+  void* stage[6];
+  size_t stage_bytes[6];
+};
+
+struct lddp_comm_s {
+  lddp_plan_t plan;
+  int nranks, rank, device;
+  void* window;          // [flags: nstrips u64][values: rows x 4 B]
+  size_t win_bytes;
+  void* peer;            // rank+1's window (IPC-opened or in-process)
+  bool peer_ipc;
+  uint64_t fills;
+};
+
+namespace {
+
+// Wavefront geometry for `cols` local columns.
+void wf_geometry(lddp_plan_s* pl, int64_t cols) {
+  pl->strip_rows = (int64_t)kWfWarps * 32 * pl->R;
+  const int64_t m = pl->desc.rows;
+  pl->nstrips = (int)((m + pl->strip_rows - 1) / pl->strip_rows);
+  pl->row0 = m - (int64_t)pl->nstrips * pl->strip_rows;
+  pl->nchunks = (int)((cols + 33 + 31) / 32);
+  pl->bnd_stride = (int64_t)pl->nchunks * 32;
+}
+
+size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
+
+lddp_status ensure_own_ws(lddp_plan_t pl, void** ws, cudaStream_t stream) {
+  if (*ws != nullptr) return LDDP_OK;
+  std::lock_guard<std::mutex> lk(pl->mu);
+  if (pl->own_ws == nullptr) {
+    CUDA_TRY(cudaMalloc(&pl->own_ws, std::max<size_t>(pl->ws_bytes, 64)));
+    CUDA_TRY(cudaMemsetAsync(pl->own_ws, 0, std::max<size_t>(pl->ws_bytes, 64), stream));
+  }
+  *ws = pl->own_ws;
+  return LDDP_OK;
+}
+
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    if (cudaGetDevice(&prev) == cudaSuccess && prev != dev) cudaSetDevice(dev);
+    else prev = -1;
+  }
+  ~DeviceGuard() {
+    if (prev >= 0) cudaSetDevice(prev);
+  }
+};
+
+// Score of an empty problem (one or both sequences empty): the boundary value.
+lddp_status write_empty_outputs(lddp_plan_t pl, const lddp_outputs* out, cudaStream_t s) {
+  const lddp_desc& d = pl->desc;
+  if (out->score != nullptr && (d.outputs & LDDP_OUT_SCORE)) {
+    if (d.func == LDDP_F_LCS) {
+      int32_t v = 0;
+      CUDA_TRY(cudaMemcpyAsync(out->score, &v, 4, cudaMemcpyHostToDevice, s));
+    } else if (d.func == LDDP_F_LEVENSHTEIN) {
+      int32_t v = (int32_t)std::max(d.rows, d.cols);
+      CUDA_TRY(cudaMemcpyAsync(out->score, &v, 4, cudaMemcpyHostToDevice, s));
+    } else if (d.func == LDDP_F_DTW) {
+      float v = (d.rows == 0 && d.cols == 0) ? 0.0f : __builtin_inff();
+      CUDA_TRY(cudaMemcpyAsync(out->score, &v, 4, cudaMemcpyHostToDevice, s));
+    }
+    // memcpy from a stack variable: make it synchronous with respect to the host
+    CUDA_TRY(cudaStreamSynchronize(s));
+  }
+  // LCS / Lev / DTW with rows > 0 and cols == 0: last_col of an empty region is empty; with
+  // rows == 0 and cols > 0 the region's last row is empty.  Nothing else to write.
+  return LDDP_OK;
+}
+
+lddp_status check_inputs(lddp_plan_t pl, const lddp_inputs* in, const lddp_outputs* out) {
+  const lddp_desc& d = pl->desc;
+  if (in == nullptr || out == nullptr) return fail(LDDP_ERR_INVALID_ARG, "inputs/outputs is NULL");
+  if (seq_func(d.func)) {
+    if ((d.rows > 0 && in->a == nullptr) || (d.cols > 0 && in->b == nullptr))
+      return fail(LDDP_ERR_INVALID_ARG, "sequence input a/b is NULL");
+  } else {
+    if (in->grid == nullptr) return fail(LDDP_ERR_INVALID_ARG, "grid input is NULL");
+    if (in->grid_pitch < d.cols) return fail(LDDP_ERR_SHAPE, "grid_pitch < cols");
+  }
+  if ((d.outputs & LDDP_OUT_SCORE) && out->score == nullptr)
+    return fail(LDDP_ERR_INVALID_ARG, "SCORE requested but outputs.score is NULL");
+  if ((d.outputs & LDDP_OUT_LAST_ROW) && out->last_row == nullptr)
+    return fail(LDDP_ERR_INVALID_ARG, "LAST_ROW requested but outputs.last_row is NULL");
+  if ((d.outputs & LDDP_OUT_LAST_COL) && out->last_col == nullptr)
+    return fail(LDDP_ERR_INVALID_ARG, "LAST_COL requested but outputs.last_col is NULL");
+  if (d.outputs & LDDP_OUT_TABLE) {
+    if (out->table == nullptr) return fail(LDDP_ERR_INVALID_ARG, "TABLE requested but outputs.table is NULL");
+    if (out->table_pitch < d.cols) return fail(LDDP_ERR_SHAPE, "table_pitch < cols");
+  }
+  return LDDP_OK;
+}
+
+void fill_common(lddp_plan_t pl, const lddp_inputs* in, const lddp_outputs* out, void* ws,
+                 FillParams& p) {
+  const lddp_desc& d = pl->desc;
+  memset(&p, 0, sizeof p);
+  p.a = in->a;
+  p.b = in->b;
+  p.grid = in->grid;
+  p.grid_pitch = in->grid_pitch;
+  p.rows = d.rows;
+  p.cols = (int32_t)d.cols;
+  p.col0 = 0;
+  p.cols_total = (int32_t)d.cols;
+  p.param_c = d.param_c;
+  p.outputs = d.outputs;
+  p.is_last_rank = 1;
+  p.score = (d.outputs & LDDP_OUT_SCORE) ? out->score : nullptr;
+  p.last_row = (d.outputs & LDDP_OUT_LAST_ROW) ? out->last_row : nullptr;
+  p.last_col = (d.outputs & LDDP_OUT_LAST_COL) ? out->last_col : nullptr;
+  p.table = (d.outputs & LDDP_OUT_TABLE) ? out->table : nullptr;
+  p.table_pitch = out->table_pitch;
+  p.ctl = ws;
+  p.prog = reinterpret_cast<uint64_t*>(static_cast<char*>(ws) + pl->off_prog);
+  p.bnd = static_cast<char*>(ws) + pl->off_bnd;
+  p.bnd_stride = pl->bnd_stride;
+  p.epoch = g_epoch.fetch_add(1) + 1;
+  p.timeout_ns = (uint64_t)env_int("LDDP_TIMEOUT_MS", 30000) * 1000000ull;
+  p.nstrips = pl->kind == 1 ? pl->nbands : pl->nstrips;
+  p.nchunks = pl->nchunks;
+  p.row0 = pl->row0;
+  p.strip_rows = pl->strip_rows;
+  p.block_cols = kPrevBW;
+  p.halo = kPrevBandRows;
+  p.nblocks = pl->nblocks;
+}
+
+lddp_status launch(lddp_plan_t pl, const FillParams& p, cudaStream_t s) {
+  cudaError_t e = cudaSuccess;
+  if (pl->kind == 0) {
+    int grid = std::min(pl->grid, p.nstrips);
+    int r = wf_dispatch(pl->desc.func, 0, pl->variant, p.table != nullptr, &p, grid, s);
+    if (r < 0) return fail(LDDP_ERR_UNSUPPORTED, "wavefront variant %d not compiled for f=%d", pl->variant, pl->desc.func);
+    e = (cudaError_t)r;
+  } else if (pl->kind == 1) {
+    const int64_t ntasks = (int64_t)pl->nblocks * pl->nbands;
+    int grid = (int)std::min<int64_t>(pl->grid, (ntasks + 7) / 8);
+    e = lddp::launch_prevrow(pl->desc.func, p, grid, s);
+  } else {
+    e = lddp::launch_invl(pl->desc.func, p, pl->grid, s);
+  }
+  if (e != cudaSuccess) return cuda_fail(e, "kernel launch");
+  return LDDP_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+int32_t lddp_abi_version(void) { return LDDP_ABI_VERSION; }
+
+const char* lddp_status_string(lddp_status s) {
+  switch (s) {
+    case LDDP_OK: return "LDDP_OK";
+    case LDDP_ERR_INVALID_ARG: return "LDDP_ERR_INVALID_ARG";
+    case LDDP_ERR_SHAPE: return "LDDP_ERR_SHAPE";
+    case LDDP_ERR_CATEGORY_MISMATCH: return "LDDP_ERR_CATEGORY_MISMATCH";
+    case LDDP_ERR_UNSUPPORTED: return "LDDP_ERR_UNSUPPORTED";
+    case LDDP_ERR_OUT_OF_MEMORY: return "LDDP_ERR_OUT_OF_MEMORY";
+    case LDDP_ERR_CUDA: return "LDDP_ERR_CUDA";
+    case LDDP_ERR_COMM: return "LDDP_ERR_COMM";
+    case LDDP_ERR_TIMEOUT: return "LDDP_ERR_TIMEOUT";
+    case LDDP_ERR_INTERNAL: return "LDDP_ERR_INTERNAL";
+  }
+  return "LDDP_ERR_UNKNOWN";
+}
+
+const char* lddp_last_error_message(void) { return g_last_error.c_str(); }
+
+lddp_status lddp_func_mask(int32_t func, uint32_t* mask) {
+  if (mask == nullptr) return fail(LDDP_ERR_INVALID_ARG, "mask is NULL");
+  uint32_t m = func_mask(func);
+  if (m == 0) return fail(LDDP_ERR_INVALID_ARG, "unknown func %d", func);
+  *mask = m;
+  return LDDP_OK;
+}
+
+lddp_status lddp_classify(uint32_t mask, int32_t* pattern) {
+  if (pattern == nullptr) return fail(LDDP_ERR_INVALID_ARG, "pattern is NULL");
+  if (mask == 0 || mask > 15) return fail(LDDP_ERR_INVALID_ARG, "contributing set must be a non-empty subset of RS(i,j)");
+  *pattern = kTable1[mask];
+  return LDDP_OK;
+}
+
+lddp_status lddp_category_covers(int32_t category, uint32_t mask, int32_t* covers) {
+  if (covers == nullptr) return fail(LDDP_ERR_INVALID_ARG, "covers is NULL");
+  if (category < 0 || category > 3) return fail(LDDP_ERR_INVALID_ARG, "unknown category %d", category);
+  if (mask == 0 || mask > 15) return fail(LDDP_ERR_INVALID_ARG, "bad mask");
+  *covers = (mask & ~category_allows(category)) == 0 ? 1 : 0;
+  return LDDP_OK;
+}
+
+lddp_status lddp_plan(const lddp_desc* desc, lddp_plan_t* out) {
+  try {
+    if (desc == nullptr || out == nullptr) return fail(LDDP_ERR_INVALID_ARG, "desc/plan is NULL");
+    *out = nullptr;
+    const lddp_desc& d = *desc;
+    const uint32_t fm = func_mask(d.func);
+    if (fm == 0) return fail(LDDP_ERR_INVALID_ARG, "unknown func %d", d.func);
+    if (d.category < 0 || d.category > 3) return fail(LDDP_ERR_INVALID_ARG, "unknown category %d", d.category);
+    if (d.rows < 0 || d.cols < 0) return fail(LDDP_ERR_SHAPE, "negative shape");
+    if (d.cols > (int64_t)0x7fff0000 || d.rows > ((int64_t)1 << 40)) return fail(LDDP_ERR_SHAPE, "shape too large");
+    if (d.outputs & ~(LDDP_OUT_SCORE | LDDP_OUT_LAST_ROW | LDDP_OUT_LAST_COL | LDDP_OUT_TABLE))
+      return fail(LDDP_ERR_INVALID_ARG, "unknown output bits 0x%x", d.outputs);
+    if ((fm & ~category_allows(d.category)) != 0)
+      return fail(LDDP_ERR_CATEGORY_MISMATCH,
+                  "category %d does not order the contributing set 0x%x of f=%d (Table I)", d.category, fm, d.func);
+    if (d.func == LDDP_F_FS_DITHER && !(d.outputs & LDDP_OUT_TABLE))
+      return fail(LDDP_ERR_INVALID_ARG, "FS_DITHER writes the output image: request LDDP_OUT_TABLE");
+    if ((d.outputs & LDDP_OUT_SCORE) &&
+        (d.func == LDDP_F_FS_DITHER || d.func == LDDP_F_DIAG_MAXPLUS))
+      return fail(LDDP_ERR_INVALID_ARG, "f=%d has no score output", d.func);
+    if ((d.outputs & LDDP_OUT_LAST_COL) && d.category == LDDP_CAT_PREV_ROW)
+      return fail(LDDP_ERR_UNSUPPORTED, "LAST_COL is not produced by the prev-row kernel");
+    if (d.func == LDDP_F_MIN_PATH3 && d.rows == 0 && d.cols > 0)
+      return fail(LDDP_ERR_SHAPE, "MIN_PATH3 needs at least one row");
+
+    lddp_plan_s* pl = new (std::nothrow) lddp_plan_s();
+    if (pl == nullptr) return fail(LDDP_ERR_OUT_OF_MEMORY, "plan allocation");
+    pl->desc = d;
+    int dev = d.device;
+    cudaDeviceProp prop;
+    cudaError_t e = cudaGetDeviceProperties(&prop, dev);
+    if (e != cudaSuccess) {
+      delete pl;
+      return cuda_fail(e, "cudaGetDeviceProperties");
+    }
+    pl->sms = prop.multiProcessorCount;
+    DeviceGuard dg(dev);
+    const bool table = (d.outputs & LDDP_OUT_TABLE) != 0;
+
+    if (d.category == LDDP_CAT_ANTI_DIAGONAL || d.category == LDDP_CAT_KNIGHT_MOVE) {
+      pl->kind = 0;
+      const bool knight = d.category == LDDP_CAT_KNIGHT_MOVE;
+      int rows = d.tile_rows > 0 ? d.tile_rows : env_int("LDDP_ROWS_PER_LANE", 0);
+      int variant;
+      if (knight) {
+        variant = (rows == 2) ? 11 : 10;
+      } else {
+        int v_env = env_int("LDDP_WF_VARIANT", -1);
+        if (v_env >= 0 && v_env < 10) variant = v_env;
+        else if (rows == 2) variant = 2;
+        else if (rows == 8) variant = 3;
+        else variant = 0;
+        if (table) variant = 0;   // TABLE mode is compiled for the default variant only
+      }
+      if (d.tile_warps != 0 && d.tile_warps != kWfWarps) {
+        delete pl;
+        return fail(LDDP_ERR_UNSUPPORTED, "tile_warps=%d (this build: %d)", d.tile_warps, kWfWarps);
+      }
+      const VariantGeom* vg = variant_geom(variant);
+      if (vg == nullptr || wf_dispatch(d.func, 2, variant, table, nullptr, 0, nullptr) < 0) {
+        delete pl;
+        return fail(LDDP_ERR_UNSUPPORTED, "no compiled wavefront kernel for f=%d category=%d variant=%d table=%d",
+                    d.func, d.category, variant, (int)table);
+      }
+      pl->variant = variant;
+      pl->R = vg->R;
+      pl->SIG = vg->SIG;
+      pl->E = vg->E;
+      pl->occupancy = wf_dispatch(d.func, 1, variant, table, nullptr, 0, nullptr);
+      if (pl->occupancy <= 0) pl->occupancy = 1;
+      wf_geometry(pl, d.cols);
+      int g = d.grid_ctas > 0 ? d.grid_ctas : env_int("LDDP_GRID_CTAS", 0);
+      pl->grid = g > 0 ? g : pl->sms * pl->occupancy;
+      pl->off_prog = 64;
+      pl->off_bnd = align_up(pl->off_prog + (size_t)std::max(pl->nstrips, 1) * 8, 256);
+      pl->ws_bytes = pl->off_bnd + (size_t)std::max(pl->nstrips, 1) * pl->bnd_stride * cell_bytes(d.func);
+    } else if (d.category == LDDP_CAT_PREV_ROW) {
+      pl->kind = 1;
+      pl->nblocks = (int)((d.cols + kPrevBW - 1) / kPrevBW);
+      pl->nbands = (int)((d.rows + kPrevBandRows - 1) / kPrevBandRows);
+      pl->bnd_stride = std::max<int64_t>(d.cols, 1);
+      pl->occupancy = 4;
+      int g = d.grid_ctas > 0 ? d.grid_ctas : env_int("LDDP_GRID_CTAS", 0);
+      pl->grid = g > 0 ? g : pl->sms * pl->occupancy;
+      pl->off_prog = 64;
+      pl->off_bnd = align_up(pl->off_prog + (size_t)std::max(pl->nblocks, 1) * 16, 256);
+      pl->ws_bytes = pl->off_bnd + (size_t)kPrevRing * pl->bnd_stride * cell_bytes(d.func);
+    } else {
+      pl->kind = 2;
+      const int64_t nd = d.rows + d.cols - 1;
+      const int64_t warps = (nd + 31) / 32;
+      const int64_t blocks = (warps + (kInvlThreads / 32) - 1) / (kInvlThreads / 32);
+      pl->grid = (int)std::max<int64_t>(1, std::min<int64_t>(blocks, (int64_t)pl->sms * 8));
+      pl->off_prog = 64;
+      pl->off_bnd = 64;
+      pl->ws_bytes = 64;
+    }
+    *out = pl;
+    return LDDP_OK;
+  } catch (...) {
+    return fail(LDDP_ERR_INTERNAL, "exception in lddp_plan");
+  }
+}
+
+lddp_status lddp_plan_destroy(lddp_plan_t pl) {
+  if (pl == nullptr) return LDDP_OK;
+  DeviceGuard dg(pl->desc.device);
+  if (pl->own_ws) cudaFree(pl->own_ws);
+  for (int k = 0; k < 6; ++k)
+    if (pl->stage[k]) cudaFree(pl->stage[k]);
+  delete pl;
+  return LDDP_OK;
+}
+
+lddp_status lddp_plan_workspace_size(lddp_plan_t pl, size_t* bytes) {
+  if (pl == nullptr || bytes == nullptr) return fail(LDDP_ERR_INVALID_ARG, "NULL argument");
+  *bytes = pl->ws_bytes;
+  return LDDP_OK;
+}
+
+lddp_status lddp_plan_describe(lddp_plan_t pl, char* buf, size_t len) {
+  if (pl == nullptr || buf == nullptr || len == 0) return fail(LDDP_ERR_INVALID_ARG, "NULL argument");
+  static const char* kinds[] = {"wavefront", "prevrow", "invl"};
+  snprintf(buf, len,
+           "{\"kernel\": \"%s\", \"variant\": %d, \"rows_per_lane\": %d, \"skew\": %d, \"extra_lag\": %d, "
+           "\"warps\": %d, \"grid\": %d, \"sms\": %d, \"occupancy\": %d, \"strip_rows\": %lld, "
+           "\"strips\": %d, \"chunks\": %d, \"blocks\": %d, \"bands\": %d, \"workspace_bytes\": %zu}",
+           kinds[pl->kind], pl->variant, pl->R, pl->SIG, pl->E,
+           pl->kind == 0 ? kWfWarps + 2 : (pl->kind == 1 ? kPrevThreads / 32 : kInvlThreads / 32), pl->grid,
+           pl->sms, pl->occupancy, (long long)pl->strip_rows, pl->nstrips, pl->nchunks, pl->nblocks, pl->nbands,
+           pl->ws_bytes);
+  return LDDP_OK;
+}
+
+lddp_status lddp_workspace_init(lddp_plan_t pl, void* ws, void* stream) {
+  if (pl == nullptr || ws == nullptr) return fail(LDDP_ERR_INVALID_ARG, "NULL argument");
+  DeviceGuard dg(pl->desc.device);
+  CUDA_TRY(cudaMemsetAsync(ws, 0, std::max<size_t>(pl->ws_bytes, 64), (cudaStream_t)stream));
+  return LDDP_OK;
+}
+
+lddp_status lddp_fill(lddp_plan_t pl, const lddp_inputs* in, const lddp_outputs* out, void* ws,
+                      void* stream) {
+  try {
+    if (pl == nullptr) return fail(LDDP_ERR_INVALID_ARG, "plan is NULL");
+    lddp_status st = check_inputs(pl, in, out);
+    if (st != LDDP_OK) return st;
+    DeviceGuard dg(pl->desc.device);
+    cudaStream_t s = (cudaStream_t)stream;
+    const lddp_desc& d = pl->desc;
+    if (d.rows == 0 || d.cols == 0) return write_empty_outputs(pl, out, s);
+    if (d.func == LDDP_F_FS_DITHER) {
+      // word-wide pixel access requirements (documented in lddp.h)
+      if ((reinterpret_cast<uintptr_t>(in->grid) & 3) || (in->grid_pitch & 3) ||
+          (reinterpret_cast<uintptr_t>(out->table) & 3) || (out->table_pitch & 3))
+        return fail(LDDP_ERR_INVALID_ARG, "FS_DITHER needs 4-byte aligned image bases and pitches");
+    }
+    st = ensure_own_ws(pl, &ws, s);
+    if (st != LDDP_OK) return st;
+    FillParams p;
+    fill_common(pl, in, out, ws, p);
+    return launch(pl, p, s);
+  } catch (...) {
+    return fail(LDDP_ERR_INTERNAL, "exception in lddp_fill");
+  }
+}
+
+lddp_status lddp_fill_host(lddp_plan_t pl, const lddp_inputs* hin, const lddp_outputs* hout,
+                           void* stream) {
+  try {
+    if (pl == nullptr) return fail(LDDP_ERR_INVALID_ARG, "plan is NULL");
+    lddp_status st = check_inputs(pl, hin, hout);
+    if (st != LDDP_OK) return st;
+    DeviceGuard dg(pl->desc.device);
+    cudaStream_t s = (cudaStream_t)stream;
+    const lddp_desc& d = pl->desc;
+    std::lock_guard<std::mutex> lk(pl->mu);
+    size_t need[6] = {0, 0, 0, 0, 0, 0};
+    if (seq_func(d.func)) {
+      need[0] = d.rows * seq_elt_bytes(d.func);
+      need[1] = d.cols * seq_elt_bytes(d.func);
+    } else {
+      need[2] = d.rows * hin->grid_pitch * grid_elt_bytes(d.func);
+    }
+    need[3] = (d.outputs & LDDP_OUT_LAST_ROW) ? d.cols * cell_bytes(d.func) : 0;
+    need[4] = (d.outputs & LDDP_OUT_LAST_COL) ? d.rows * cell_bytes(d.func) : 0;
+    need[5] = (d.outputs & LDDP_OUT_TABLE) ? d.rows * hout->table_pitch * table_elt_bytes(d.func) + 16 : 16;
+    for (int k = 0; k < 6; ++k) {
+      if (need[k] > pl->stage_bytes[k]) {
+        if (pl->stage[k]) cudaFree(pl->stage[k]);
+        pl->stage[k] = nullptr;
+        pl->stage_bytes[k] = 0;
+        CUDA_TRY(cudaMalloc(&pl->stage[k], need[k]));
+        pl->stage_bytes[k] = need[k];
+      }
+    }
+    lddp_inputs din = *hin;
+    lddp_outputs dout = *hout;
+    if (need[0]) { CUDA_TRY(cudaMemcpyAsync(pl->stage[0], hin->a, need[0], cudaMemcpyHostToDevice, s)); din.a = pl->stage[0]; }
+    if (need[1]) { CUDA_TRY(cudaMemcpyAsync(pl->stage[1], hin->b, need[1], cudaMemcpyHostToDevice, s)); din.b = pl->stage[1]; }
+    if (need[2]) { CUDA_TRY(cudaMemcpyAsync(pl->stage[2], hin->grid, need[2], cudaMemcpyHostToDevice, s)); din.grid = pl->stage[2]; }
+    char* score_dev = static_cast<char*>(pl->stage[5]) + ((d.outputs & LDDP_OUT_TABLE) ? need[5] - 16 : 0);
+    dout.score = hout->score ? score_dev : nullptr;
+    dout.last_row = need[3] ? pl->stage[3] : nullptr;
+    dout.last_col = need[4] ? pl->stage[4] : nullptr;
+    dout.table = (d.outputs & LDDP_OUT_TABLE) ? pl->stage[5] : nullptr;
+    void* ws = nullptr;
+    st = ensure_own_ws(pl, &ws, s);
+    if (st != LDDP_OK) return st;
+    if (d.rows == 0 || d.cols == 0) {
+      st = write_empty_outputs(pl, &dout, s);
+    } else {
+      FillParams p;
+      fill_common(pl, &din, &dout, ws, p);
+      st = launch(pl, p, s);
+    }
+    if (st != LDDP_OK) return st;
+    if (hout->score && (d.outputs & LDDP_OUT_SCORE))
+      CUDA_TRY(cudaMemcpyAsync(hout->score, score_dev, cell_bytes(d.func), cudaMemcpyDeviceToHost, s));
+    if (need[3]) CUDA_TRY(cudaMemcpyAsync(hout->last_row, pl->stage[3], need[3], cudaMemcpyDeviceToHost, s));
+    if (need[4]) CUDA_TRY(cudaMemcpyAsync(hout->last_col, pl->stage[4], need[4], cudaMemcpyDeviceToHost, s));
+    if (d.outputs & LDDP_OUT_TABLE)
+      CUDA_TRY(cudaMemcpyAsync(hout->table, pl->stage[5], need[5] - 16, cudaMemcpyDeviceToHost, s));
+    CUDA_TRY(cudaStreamSynchronize(s));
+    return lddp_status_check(pl, ws, stream);
+  } catch (...) {
+    return fail(LDDP_ERR_INTERNAL, "exception in lddp_fill_host");
+  }
+}
+
+lddp_status lddp_status_check(lddp_plan_t pl, void* ws, void* stream) {
+  if (pl == nullptr) return fail(LDDP_ERR_INVALID_ARG, "plan is NULL");
+  DeviceGuard dg(pl->desc.device);
+  cudaStream_t s = (cudaStream_t)stream;
+  CUDA_TRY(cudaStreamSynchronize(s));
+  if (ws == nullptr) ws = pl->own_ws;
+  if (ws == nullptr) return LDDP_OK;
+  lddp::Control c;
+  CUDA_TRY(cudaMemcpy(&c, ws, sizeof c, cudaMemcpyDeviceToHost));
+  if (c.status != 0) {
+    CUDA_TRY(cudaMemset(ws, 0, sizeof c));   // make the workspace usable again
+    return fail((lddp_status)c.status, "device watchdog: a dependency wait exceeded LDDP_TIMEOUT_MS");
+  }
+  return LDDP_OK;
+}
+
+// ------------------------------------------------------------------------------ multi-GPU
+lddp_status lddp_comm_create(lddp_plan_t pl, int32_t nranks, int32_t rank, lddp_comm_t* out) {
+  if (pl == nullptr || out == nullptr) return fail(LDDP_ERR_INVALID_ARG, "NULL argument");
+  if (nranks < 1 || rank < 0 || rank >= nranks) return fail(LDDP_ERR_INVALID_ARG, "bad rank %d / %d", rank, nranks);
+  if (pl->kind != 0 || pl->desc.category != LDDP_CAT_ANTI_DIAGONAL)
+    return fail(LDDP_ERR_UNSUPPORTED, "multi-GPU column strips: anti-diagonal category only in this build");
+  if (pl->desc.cols < nranks) return fail(LDDP_ERR_SHAPE, "cols < nranks");
+  DeviceGuard dg(pl->desc.device);
+  lddp_comm_s* c = new (std::nothrow) lddp_comm_s();
+  if (c == nullptr) return fail(LDDP_ERR_OUT_OF_MEMORY, "comm allocation");
+  c->plan = pl;
+  c->nranks = nranks;
+  c->rank = rank;
+  c->device = pl->desc.device;
+  c->win_bytes = align_up((size_t)std::max(pl->nstrips, 1) * 8, 256) + (size_t)std::max<int64_t>(pl->desc.rows, 1) * 4;
+  cudaError_t e = cudaMalloc(&c->window, c->win_bytes);
+  if (e == cudaSuccess) e = cudaMemset(c->window, 0, c->win_bytes);
+  if (e != cudaSuccess) {
+    delete c;
+    return cuda_fail(e, "window allocation");
+  }
+  *out = c;
+  return LDDP_OK;
+}
+
+lddp_status lddp_comm_handle(lddp_comm_t c, uint8_t handle[LDDP_COMM_HANDLE_BYTES]) {
+  if (c == nullptr || handle == nullptr) return fail(LDDP_ERR_INVALID_ARG, "NULL argument");
+  static_assert(sizeof(cudaIpcMemHandle_t) <= LDDP_COMM_HANDLE_BYTES, "IPC handle size");
+  DeviceGuard dg(c->device);
+  cudaIpcMemHandle_t h;
+  cudaError_t e = cudaIpcGetMemHandle(&h, c->window);
+  if (e != cudaSuccess) return fail(LDDP_ERR_COMM, "cudaIpcGetMemHandle: %s", cudaGetErrorString(e));
+  memset(handle, 0, LDDP_COMM_HANDLE_BYTES);
+  memcpy(handle, &h, sizeof h);
+  return LDDP_OK;
+}
+
+lddp_status lddp_comm_connect(lddp_comm_t c, const uint8_t next_handle[LDDP_COMM_HANDLE_BYTES]) {
+  if (c == nullptr) return fail(LDDP_ERR_INVALID_ARG, "comm is NULL");
+  if (c->rank == c->nranks - 1 || next_handle == nullptr) {
+    c->peer = nullptr;
+    return LDDP_OK;
+  }
+  DeviceGuard dg(c->device);
+  cudaIpcMemHandle_t h;
+  memcpy(&h, next_handle, sizeof h);
+  void* p = nullptr;
+  cudaError_t e = cudaIpcOpenMemHandle(&p, h, cudaIpcMemLazyEnablePeerAccess);
+  if (e != cudaSuccess) return fail(LDDP_ERR_COMM, "cudaIpcOpenMemHandle: %s", cudaGetErrorString(e));
+  c->peer = p;
+  c->peer_ipc = true;
+  return LDDP_OK;
+}
+
+lddp_status lddp_comm_connect_local(lddp_comm_t c, lddp_comm_t next) {
+  if (c == nullptr) return fail(LDDP_ERR_INVALID_ARG, "comm is NULL");
+  if (next == nullptr) {
+    c->peer = nullptr;
+    return LDDP_OK;
+  }
+  if (next->device != c->device) {
+    DeviceGuard dg(c->device);
+    int ok = 0;
+    cudaDeviceCanAccessPeer(&ok, c->device, next->device);
+    if (!ok) return fail(LDDP_ERR_COMM, "device %d cannot access peer %d", c->device, next->device);
+    cudaError_t e = cudaDeviceEnablePeerAccess(next->device, 0);
+    if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled)
+      return fail(LDDP_ERR_COMM, "cudaDeviceEnablePeerAccess: %s", cudaGetErrorString(e));
+    cudaGetLastError();
+  }
+  c->peer = next->window;
+  c->peer_ipc = false;
+  return LDDP_OK;
+}
+
+lddp_status lddp_comm_destroy(lddp_comm_t c) {
+  if (c == nullptr) return LDDP_OK;
+  DeviceGuard dg(c->device);
+  if (c->peer_ipc && c->peer) cudaIpcCloseMemHandle(c->peer);
+  if (c->window) cudaFree(c->window);
+  delete c;
+  return LDDP_OK;
+}
+
+lddp_status lddp_fill_multi(lddp_plan_t pl, const lddp_inputs* in, const lddp_outputs* out,
+                            void* ws, lddp_comm_t c, void* stream) {
+  try {
+    if (pl == nullptr || c == nullptr) return fail(LDDP_ERR_INVALID_ARG, "NULL argument");
+    if (c->plan != pl) return fail(LDDP_ERR_INVALID_ARG, "comm was created for another plan");
+    lddp_status st = check_inputs(pl, in, out);
+    if (st != LDDP_OK) return st;
+    if (c->rank < c->nranks - 1 && c->peer == nullptr)
+      return fail(LDDP_ERR_COMM, "rank %d is not connected to rank %d", c->rank, c->rank + 1);
+    DeviceGuard dg(pl->desc.device);
+    cudaStream_t s = (cudaStream_t)stream;
+    const lddp_desc& d = pl->desc;
+    if (d.rows == 0) return LDDP_OK;
+    st = ensure_own_ws(pl, &ws, s);
+    if (st != LDDP_OK) return st;
+    const int64_t n = d.cols;
+    const int64_t c0 = (int64_t)c->rank * n / c->nranks;
+    const int64_t c1 = (int64_t)(c->rank + 1) * n / c->nranks;
+    FillParams p;
+    fill_common(pl, in, out, ws, p);
+    p.cols = (int32_t)(c1 - c0);
+    p.col0 = (int32_t)c0;
+    p.cols_total = (int32_t)n;
+    p.nchunks = (int)((p.cols + 33 + 31) / 32);
+    p.bnd_stride = (int64_t)p.nchunks * 32;
+    const bool last = c->rank == c->nranks - 1;
+    p.is_last_rank = last ? 1 : 0;
+    if (p.last_row) p.last_row = static_cast<char*>(p.last_row) + c0 * cell_bytes(d.func);
+    if (!last) {
+      p.score = nullptr;
+      p.last_col = nullptr;
+      p.table = nullptr;
+    }
+    if (p.table) return fail(LDDP_ERR_UNSUPPORTED, "TABLE output is not supported by lddp_fill_multi");
+    const size_t flags_bytes = align_up((size_t)std::max(pl->nstrips, 1) * 8, 256);
+    c->fills += 1;
+    p.wepoch = c->fills;
+    if (c->rank > 0) {
+      p.lflag_in = reinterpret_cast<const uint64_t*>(c->window);
+      p.lcol_in = static_cast<const char*>(c->window) + flags_bytes;
+    }
+    if (!last) {
+      p.rflag_out = reinterpret_cast<uint64_t*>(c->peer);
+      p.rcol_out = static_cast<char*>(c->peer) + flags_bytes;
+    }
+    return launch(pl, p, s);
+  } catch (...) {
+    return fail(LDDP_ERR_INTERNAL, "exception in lddp_fill_multi");
+  }
+}
+
+}  // extern "C"

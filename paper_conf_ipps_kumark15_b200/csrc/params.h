@@ -1,0 +1,63 @@
+// params.h -- kernel parameter block and launch entry points shared by the C-ABI layer
+// (lddp_api.cpp, host C++) and the CUDA translation units.  Internal to liblddp.so.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace lddp {
+
+struct FillParams {
+  // problem (local to this rank for multi-GPU)
+  const void* a;            // LCS/Lev: uint8[rows], DTW: float[rows]
+  const void* b;            // LCS/Lev: uint8[cols_total], DTW: float[cols_total] (global)
+  const void* grid;         // FS uint8 / int32 grid, rows x cols
+  int64_t grid_pitch;       // elements
+  int64_t rows;             // m / H
+  int32_t cols;             // local number of f-evaluated columns
+  int32_t col0;             // global column of local column 0 (multi-GPU), else 0
+  int32_t cols_total;       // global number of columns
+  int32_t param_c;
+  uint32_t outputs;         // LDDP_OUT_* bits
+  int32_t is_last_rank;     // 1 on single GPU / last rank (owns score + last_col)
+  // outputs (device pointers, NULL if not requested)
+  void* score;
+  void* last_row;           // already offset by col0 on multi-GPU
+  void* last_col;
+  void* table;
+  int64_t table_pitch;
+  // workspace
+  void* ctl;                // lddp::Control*
+  uint64_t* prog;           // per strip / band progress flags (epoch << 32 | count)
+  void* bnd;                // boundary rows between strips / bands
+  int64_t bnd_stride;       // elements per strip row in bnd
+  uint64_t epoch;           // workspace epoch (progress flags)
+  uint64_t wepoch;          // multi-GPU window epoch (rank-consistent)
+  uint64_t timeout_ns;
+  // geometry
+  int32_t nstrips;          // strips (anti-diag / knight) or bands (prev-row)
+  int32_t nchunks;          // link chunks per strip (anti-diag / knight)
+  int64_t row0;             // global row of strip 0's first row (<= 0: bottom-aligned strips)
+  int64_t strip_rows;       // rows per strip / band
+  // prev-row category
+  int32_t block_cols;       // columns owned per CTA
+  int32_t halo;             // trapezoid halo (= band rows)
+  int32_t nblocks;          // column blocks
+  // multi-GPU window (left boundary in, right column out)
+  const void* lcol_in;      // my window: rows values of rank g-1's right column
+  const uint64_t* lflag_in; // my window flags, one per strip
+  void* rcol_out;           // rank g+1's window (peer pointer) or NULL
+  uint64_t* rflag_out;      // rank g+1's window flags (peer pointer) or NULL
+};
+
+// Launch entry points (one per category family).  Return cudaError_t of the launch.
+cudaError_t launch_wavefront(int func, int category, const FillParams& p, int rows_per_lane,
+                             int warps, int grid, cudaStream_t stream);
+cudaError_t launch_prevrow(int func, const FillParams& p, int grid, cudaStream_t stream);
+cudaError_t launch_invl(int func, const FillParams& p, int grid, cudaStream_t stream);
+
+// Per-kernel occupancy query (blocks per SM) for the chosen configuration.
+int wavefront_blocks_per_sm(int func, int category, int rows_per_lane, int warps);
+size_t wavefront_smem_bytes(int func, int category, int rows_per_lane, int warps);
+bool wavefront_supported(int func, int category, int rows_per_lane, int warps);
+
+}  // namespace lddp

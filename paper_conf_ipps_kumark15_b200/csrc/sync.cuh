@@ -1,0 +1,115 @@
+// sync.cuh -- device synchronisation primitives of the persistent LDDP kernels (sm_100a).
+//
+// * mbarrier producer/consumer rings between warps of one CTA (intra-strip handoff);
+// * epoch-tagged release/acquire progress flags in global memory between CTAs (strip handoff,
+//   SURVEY §8(a3)) and between GPUs over NVLink (system scope, §8(e));
+// * a watchdog: every dependency wait is bounded (globaltimer), so a protocol bug reports
+//   LDDP_ERR_TIMEOUT through the workspace status word instead of hanging the device.
+#pragma once
+#include <cstdint>
+
+namespace lddp {
+
+struct Control {                 // workspace header (device), zeroed by lddp_workspace_init
+  unsigned int claim;            // next strip / band to claim (persistent scheduler)
+  unsigned int done;             // CTAs finished (last one resets claim / done)
+  unsigned int status;           // 0 or lddp_status of a device-side failure
+  unsigned int abort;            // set on watchdog expiry: every wait gives up
+  unsigned int pad[12];
+};
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.release.cta.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ bool mbar_try_wait(uint64_t* bar, uint32_t parity) {
+  uint32_t ok;
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "mbarrier.try_wait.parity.acquire.cta.shared::cta.b64 p, [%1], %2;\n\t"
+      "selp.u32 %0, 1, 0, p;\n\t}"
+      : "=r"(ok)
+      : "r"(smem_u32(bar)), "r"(parity)
+      : "memory");
+  return ok != 0;
+}
+
+__device__ __forceinline__ uint64_t globaltimer_ns() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+
+__device__ __forceinline__ uint64_t ld_acquire_gpu(const uint64_t* p) {
+  uint64_t v;
+  asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ uint64_t ld_acquire_sys(const uint64_t* p) {
+  uint64_t v;
+  asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_gpu(uint64_t* p, uint64_t v) {
+  asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ void st_release_sys(uint64_t* p, uint64_t v) {
+  asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ unsigned ld_volatile_u32(const unsigned* p) {
+  return *reinterpret_cast<const volatile unsigned*>(p);
+}
+
+// Watchdog bookkeeping for one waiting thread.
+struct Watch {
+  uint64_t t0;
+  uint32_t spins;
+  __device__ __forceinline__ Watch() : t0(0), spins(0) {}
+  // Returns false if the wait must be abandoned (abort flag or timeout).
+  __device__ __forceinline__ bool tick(Control* ctl, uint64_t timeout_ns) {
+    ++spins;
+    if (spins < 32) return true;
+    __nanosleep(spins < 1024 ? 32 : 256);
+    if ((spins & 255) != 0) return true;
+    if (ld_volatile_u32(&ctl->abort)) return false;
+    uint64_t now = globaltimer_ns();
+    if (t0 == 0) { t0 = now; return true; }
+    if (now - t0 > timeout_ns) {
+      atomicCAS(&ctl->status, 0u, 8u /* LDDP_ERR_TIMEOUT */);
+      atomicExch(&ctl->abort, 1u);
+      return false;
+    }
+    return true;
+  }
+};
+
+// Wait until an epoch-tagged flag (epoch << 32 | count) reaches `target`.
+template <bool kSys>
+__device__ __forceinline__ bool wait_flag(const uint64_t* flag, uint64_t target, Control* ctl,
+                                          uint64_t timeout_ns) {
+  Watch w;
+  while (true) {
+    uint64_t v = kSys ? ld_acquire_sys(flag) : ld_acquire_gpu(flag);
+    if (v >= target) return true;
+    if (!w.tick(ctl, timeout_ns)) return false;
+  }
+}
+
+// Bounded mbarrier wait (phase parity).
+__device__ __forceinline__ bool mbar_wait(uint64_t* bar, uint32_t parity, Control* ctl,
+                                          uint64_t timeout_ns) {
+  if (mbar_try_wait(bar, parity)) return true;
+  Watch w;
+  while (!mbar_try_wait(bar, parity)) {
+    if (!w.tick(ctl, timeout_ns)) return false;
+  }
+  return true;
+}
+
+}  // namespace lddp
