@@ -201,15 +201,21 @@ void wf_geometry(lddp_plan_s* pl, int64_t cols) {
 
 size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
 
-lddp_status ensure_own_ws(lddp_plan_t pl, void** ws, cudaStream_t stream) {
+// Caller must hold pl->mu.
+lddp_status ensure_own_ws_locked(lddp_plan_t pl, void** ws, cudaStream_t stream) {
   if (*ws != nullptr) return LDDP_OK;
-  std::lock_guard<std::mutex> lk(pl->mu);
   if (pl->own_ws == nullptr) {
     CUDA_TRY(cudaMalloc(&pl->own_ws, std::max<size_t>(pl->ws_bytes, 64)));
     CUDA_TRY(cudaMemsetAsync(pl->own_ws, 0, std::max<size_t>(pl->ws_bytes, 64), stream));
   }
   *ws = pl->own_ws;
   return LDDP_OK;
+}
+
+lddp_status ensure_own_ws(lddp_plan_t pl, void** ws, cudaStream_t stream) {
+  if (*ws != nullptr) return LDDP_OK;
+  std::lock_guard<std::mutex> lk(pl->mu);
+  return ensure_own_ws_locked(pl, ws, stream);
 }
 
 struct DeviceGuard {
@@ -301,6 +307,15 @@ void fill_common(lddp_plan_t pl, const lddp_inputs* in, const lddp_outputs* out,
   p.block_cols = kPrevBW;
   p.halo = kPrevBandRows;
   p.nblocks = pl->nblocks;
+  // debug trace buffer: LDDP_TRACE=<device pointer as decimal>:<chunks per row>
+  if (const char* tr = getenv("LDDP_TRACE")) {
+    unsigned long long ptr = 0;
+    int chunks = 0;
+    if (sscanf(tr, "%llu:%d", &ptr, &chunks) == 2) {
+      p.trace = reinterpret_cast<uint64_t*>(ptr);
+      p.trace_chunks = chunks;
+    }
+  }
 }
 
 lddp_status launch(lddp_plan_t pl, const FillParams& p, cudaStream_t s) {
@@ -575,7 +590,7 @@ lddp_status lddp_fill_host(lddp_plan_t pl, const lddp_inputs* hin, const lddp_ou
     dout.last_col = need[4] ? pl->stage[4] : nullptr;
     dout.table = (d.outputs & LDDP_OUT_TABLE) ? pl->stage[5] : nullptr;
     void* ws = nullptr;
-    st = ensure_own_ws(pl, &ws, s);
+    st = ensure_own_ws_locked(pl, &ws, s);   // pl->mu is held
     if (st != LDDP_OK) return st;
     if (d.rows == 0 || d.cols == 0) {
       st = write_empty_outputs(pl, &dout, s);

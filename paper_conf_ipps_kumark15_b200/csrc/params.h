@@ -47,6 +47,9 @@ struct FillParams {
   const uint64_t* lflag_in; // my window flags, one per strip
   void* rcol_out;           // rank g+1's window (peer pointer) or NULL
   uint64_t* rflag_out;      // rank g+1's window flags (peer pointer) or NULL
+  // debug trace (env LDDP_TRACE): globaltimer stamps per (strip, warp, chunk), or NULL
+  uint64_t* trace;
+  int32_t trace_chunks;     // chunks per (strip, warp) row of the trace
 };
 
 // Launch entry points (one per category family).  Return cudaError_t of the launch.

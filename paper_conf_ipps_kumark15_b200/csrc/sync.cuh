@@ -56,6 +56,12 @@ __device__ __forceinline__ uint64_t ld_acquire_sys(const uint64_t* p) {
   asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
   return v;
 }
+__device__ __forceinline__ uint64_t ld_relaxed_gpu(const uint64_t* p) {
+  uint64_t v;
+  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void fence_acq_rel_gpu() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
 __device__ __forceinline__ void st_release_gpu(uint64_t* p, uint64_t v) {
   asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
@@ -67,6 +73,10 @@ __device__ __forceinline__ unsigned ld_volatile_u32(const unsigned* p) {
 }
 
 // Watchdog bookkeeping for one waiting thread.
+// kSleep: back off with __nanosleep between polls of a global flag (spares L2 bandwidth);
+// mbarrier waits do not sleep (try_wait already suspends the warp in hardware until the
+// phase flips or a short time limit expires).
+template <bool kSleep = true>
 struct Watch {
   uint64_t t0;
   uint32_t spins;
@@ -74,9 +84,11 @@ struct Watch {
   // Returns false if the wait must be abandoned (abort flag or timeout).
   __device__ __forceinline__ bool tick(Control* ctl, uint64_t timeout_ns) {
     ++spins;
-    if (spins < 32) return true;
-    __nanosleep(spins < 1024 ? 32 : 256);
-    if ((spins & 255) != 0) return true;
+    if (kSleep) {
+      if (spins < 64) return true;
+      __nanosleep(spins < 4096 ? 20 : 200);
+    }
+    if ((spins & 1023) != 0) return true;
     if (ld_volatile_u32(&ctl->abort)) return false;
     uint64_t now = globaltimer_ns();
     if (t0 == 0) { t0 = now; return true; }
@@ -93,10 +105,26 @@ struct Watch {
 template <bool kSys>
 __device__ __forceinline__ bool wait_flag(const uint64_t* flag, uint64_t target, Control* ctl,
                                           uint64_t timeout_ns) {
-  Watch w;
+  Watch<true> w;
   while (true) {
     uint64_t v = kSys ? ld_acquire_sys(flag) : ld_acquire_gpu(flag);
     if (v >= target) return true;
+    if (!w.tick(ctl, timeout_ns)) return false;
+  }
+}
+
+// Acquire pattern without an L1 invalidation per poll: relaxed polls, then one acq_rel fence
+// once the released value is observed.  Returns the observed flag in `seen`.
+__device__ __forceinline__ bool wait_flag_relaxed(const uint64_t* flag, uint64_t target, Control* ctl,
+                                                  uint64_t timeout_ns, uint64_t& seen) {
+  Watch<true> w;
+  while (true) {
+    uint64_t v = ld_relaxed_gpu(flag);
+    if (v >= target) {
+      seen = v;
+      fence_acq_rel_gpu();
+      return true;
+    }
     if (!w.tick(ctl, timeout_ns)) return false;
   }
 }
@@ -105,7 +133,7 @@ __device__ __forceinline__ bool wait_flag(const uint64_t* flag, uint64_t target,
 __device__ __forceinline__ bool mbar_wait(uint64_t* bar, uint32_t parity, Control* ctl,
                                           uint64_t timeout_ns) {
   if (mbar_try_wait(bar, parity)) return true;
-  Watch w;
+  Watch<false> w;
   while (!mbar_try_wait(bar, parity)) {
     if (!w.tick(ctl, timeout_ns)) return false;
   }

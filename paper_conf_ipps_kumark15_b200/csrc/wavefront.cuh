@@ -25,6 +25,7 @@
 //    global memory.
 #pragma once
 #include <cstdint>
+#include <cstring>
 #include "cellfn.cuh"
 #include "params.h"
 #include "sync.cuh"
@@ -32,12 +33,10 @@
 namespace lddp {
 
 constexpr int kChunk = 32;  // link chunk = 32 entries = one per lane
+constexpr int kUnroll = 8;  // steps per unrolled loop body
+constexpr int kBatch = 4;   // chunks moved per loader / storer round trip
+constexpr int kBRing = 4096; // column-context ring (entries); index = (column + 32) & (kBRing - 1)
 
-template <class F>
-struct LinkEntry {
-  typename F::T v;
-  typename F::ColCtx cc;
-};
 
 template <class F, int R, int SIG, int E, int W, bool TABLE>
 struct Wave {
@@ -46,14 +45,12 @@ struct Wave {
   using RC = typename F::RowCtx;
   using G = typename F::GridT;
   using O = typename F::OutT;
-  using Entry = LinkEntry<F>;
   static constexpr int C = kChunk;
   static constexpr int D = R * SIG + E;      // per-lane lag in steps
-  static constexpr int NS = 8;               // ring slots per link
+  static constexpr int NS = 16;              // ring slots per link
   static constexpr int HV = SIG + 1;         // value history depth per row
   static constexpr int HC = SIG > 0 ? SIG : 1;  // column-context history depth per row
   static constexpr int FV = SIG + E + 1;     // FIFO depth (values from the lane above)
-  static constexpr int FC = SIG + E;         // FIFO depth (column contexts)
   static constexpr int kThreads = (W + 2) * 32;
   static constexpr int TAU0 = -32 - SIG - E; // step at which lane 31 injects top entry q = 0
   static_assert(E >= 1, "need at least one step of shuffle slack");
@@ -61,9 +58,10 @@ struct Wave {
   static_assert(SIG + E >= 2 || !(F::kMask & NB_UR), "UR of row 0 must be at least one step old");
 
   struct Smem {
-    Entry link[W + 1][NS][C];
+    alignas(16) T link[W + 1][NS][C];
     uint64_t full[W + 1][NS];
     uint64_t empty[W + 1][NS];
+    typename F::ColCtx bring[kBRing];   // column contexts staged by the loader
     uint64_t bar;        // CTA barrier (abort-aware)
     int strip;
   };
@@ -79,6 +77,19 @@ __device__ __forceinline__ bool cta_sync(uint64_t* bar, uint32_t& phase, Control
   return ok;
 }
 
+template <class T>
+__device__ __forceinline__ T bits_to(uint32_t x) {
+  T t;
+  memcpy(&t, &x, sizeof(T));
+  return t;
+}
+template <class T>
+__device__ __forceinline__ uint32_t to_bits(T t) {
+  uint32_t x;
+  memcpy(&x, &t, sizeof(T));
+  return x;
+}
+
 template <class F, int R, int SIG, int E, int W, bool TABLE>
 struct WaveCompute {
   using WV = Wave<F, R, SIG, E, W, TABLE>;
@@ -87,110 +98,175 @@ struct WaveCompute {
   using RC = typename WV::RC;
   using G = typename WV::G;
   using O = typename WV::O;
-  using Entry = typename WV::Entry;
-  static constexpr int C = WV::C, D = WV::D, HV = WV::HV, HC = WV::HC, FV = WV::FV, FC = WV::FC;
+  static constexpr int C = WV::C, D = WV::D, HV = WV::HV, HC = WV::HC, FV = WV::FV;
+  static_assert(sizeof(T) == 4, "link values are 32-bit");
 
   T hist[R][HV];   // hist[r][d] = value of row r at step tau-1-d
-  CC hcc[R][HC];   // hcc[r][d]  = column context of row r at step tau-1-d
+  CC hcc[R][HC];   // hcc[r][d]  = column context of row r at step tau-1-d (SIG > 0)
   T fifo[FV];      // fifo[d]    = value received from the lane above at the end of step tau-1-d
-  CC fcc[FC > 0 ? FC : 1];
   RC rc[R];
-  int64_t irow[R];
+  int irow[R];     // global row of each lane-row (may be < 0 in strip 0: virtual rows)
+  T leftv[R];      // value of column -1 of the row (initialisation, or rank g-1's column)
+  T rightv[R];     // value of column n of the row (only read through UR)
+  bool vtop[R];    // the lane-row is strip 0's virtual row -1 (holds the top initialisation)
+  bool rvalid[R];  // 0 <= row < m
+  T rlast[R];      // the row's value at column n-1 (captured in boundary chunks)
 
-  template <bool CHECKED>
+  // Loads for the 8 steps starting at tau0: row 0's column context and each row's grid input.
+  const CC* bring;  // shared-memory column-context ring (staged by the loader warp)
+
+  template <int MODE, int U>
+  __device__ __forceinline__ void prefetch(const FillParams& p, const int lane_off, const int tau0,
+                                           CC (&cc)[U], G (&g)[R][U]) const {
+    const int n = p.cols;
+#pragma unroll
+    for (int su = 0; su < U; ++su) {
+      const int c0 = tau0 + su - lane_off;
+      cc[su] = bring[(c0 + 32) & (kBRing - 1)];
+#pragma unroll
+      for (int r = 0; r < R; ++r) {
+        const int c = c0 - r * SIG;
+        if (!F::kGridIn) {
+          g[r][su] = G(0);
+        } else if (MODE == 2) {
+          g[r][su] = (rvalid[r] && (unsigned)c < (unsigned)n) ? F::load(p, irow[r], c) : G(0);
+        } else if (MODE == 1) {
+          g[r][su] = rvalid[r] ? F::load(p, irow[r], c) : G(0);
+        } else {
+          g[r][su] = F::load(p, irow[r], c);
+        }
+      }
+    }
+  }
+
+  // One chunk of C steps.  MODE 0: steady (every cell interior); MODE 1: steady + strip 0's
+  // virtual row -1 (one select per cell); MODE 2: checked (boundary columns, virtual rows,
+  // output columns).
+  // Per step: R cells, one __shfl_sync (the bottom row value, lane k -> k+1, lane 31 -> 0
+  // injecting the warp's top link), one L1-cached load of row 0's column context.  Lane 31's
+  // top-link values and bottom-link values move 8 steps at a time as two 128-bit smem ops.
+  template <int MODE>
   __device__ __forceinline__ void chunk(const FillParams& p, const int lane, const int tau_k,
-                                        const Entry* __restrict__ top, Entry* __restrict__ bot,
+                                        const T* __restrict__ top, T* __restrict__ bot,
                                         const bool has_bot) {
+    // the checked body is executed only a few chunks per strip: keep its code small
+    constexpr int U = kUnroll;
+    constexpr bool CHECKED = MODE == 2;
     const int n = p.cols;
     const int lane_off = lane * D;
+    // Row 0's column contexts and every row's grid inputs are loaded one 8-step block ahead,
+    // so the L1 / L2 latency of those loads is off the per-step critical path.
+    CC ccc[U];
+    G gcur[R][U];
+    prefetch<MODE, U>(p, lane_off, tau_k, ccc, gcur);
+#pragma unroll 1
+    for (int sb = 0; sb < C; sb += U) {
+      CC ccn[U];
+      G gnxt[R][U];
+      if (sb + U < C) prefetch<MODE, U>(p, lane_off, tau_k + sb + U, ccn, gnxt);
+      T tv[U];
+      if (U == 8) {
+        const uint4 q0 = reinterpret_cast<const uint4*>(top + sb)[0];
+        const uint4 q1 = reinterpret_cast<const uint4*>(top + sb)[1];
+        tv[0] = bits_to<T>(q0.x); tv[1 % U] = bits_to<T>(q0.y); tv[2 % U] = bits_to<T>(q0.z); tv[3 % U] = bits_to<T>(q0.w);
+        tv[4 % U] = bits_to<T>(q1.x); tv[5 % U] = bits_to<T>(q1.y); tv[6 % U] = bits_to<T>(q1.z); tv[7 % U] = bits_to<T>(q1.w);
+      } else {
 #pragma unroll
-    for (int st = 0; st < C; ++st) {
-      const int tau = tau_k + st;
-      T nw[R];
-      CC ncc[R];
+        for (int su = 0; su < U; ++su) tv[su] = top[sb + su];
+      }
+      T bv[U];
 #pragma unroll
-      for (int r = 0; r < R; ++r) {
-        const int c = tau - lane_off - r * SIG;
-        T L = hist[r][0], U, UL, UR;
-        CC cc;
-        if (r == 0) {
-          U = fifo[SIG + E - 1];
-          UL = fifo[SIG + E];
-          UR = fifo[(SIG + E >= 2) ? SIG + E - 2 : 0];
-          cc = fcc[SIG + E - 1];
-        } else {
-          if (SIG == 0) {
-            U = nw[r - 1];
-            cc = ncc[r - 1];
+      for (int su = 0; su < U; ++su) {
+        const int tau = tau_k + sb + su;
+        T nw[R];
+        CC ncc[R];
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+          const int c = tau - lane_off - r * SIG;
+          T L = hist[r][0], U, UL, UR;
+          CC cc;
+          if (r == 0) {
+            U = fifo[SIG + E - 1];
+            UL = fifo[SIG + E];
+            UR = fifo[(SIG + E >= 2) ? SIG + E - 2 : 0];
+            cc = ccc[su];
           } else {
-            U = hist[r - 1][SIG > 0 ? SIG - 1 : 0];
-            cc = hcc[r - 1][SIG > 0 ? SIG - 1 : 0];
-          }
-          UL = hist[r - 1][SIG];
-          UR = hist[r - 1][SIG >= 2 ? SIG - 2 : 0];
-        }
-        G g = G(0);
-        if (F::kGridIn) {
-          if (CHECKED) {
-            if (c >= 0 && c < n && irow[r] >= 0) g = F::load(p, irow[r], c);
-          } else {
-            g = F::load(p, irow[r], c);
-          }
-        }
-        O o;
-        T v = F::f(L, UL, U, UR, rc[r], cc, g, irow[r], c + p.col0, p.param_c, o);
-        if (CHECKED) {
-          if (c == -1) {
-            if (p.lcol_in != nullptr) {
-              if (irow[r] >= 0) v = __ldcg(static_cast<const T*>(p.lcol_in) + irow[r]);
+            if (SIG == 0) {
+              U = nw[r - 1];
+              cc = ncc[0];
             } else {
-              v = F::left(p, irow[r]);
+              U = hist[r - 1][SIG > 0 ? SIG - 1 : 0];
+              cc = hcc[r - 1][SIG > 0 ? SIG - 1 : 0];
             }
+            UL = hist[r - 1][SIG];
+            UR = hist[r - 1][SIG >= 2 ? SIG - 2 : 0];
           }
-          if (c == n) v = F::right(p, irow[r]);
-          if (irow[r] == -1) v = F::top(p, c + p.col0);
-          if (c >= 0 && c < n && irow[r] >= 0) {
-            if (TABLE) static_cast<O*>(p.table)[irow[r] * p.table_pitch + c] = o;
-            if (c == n - 1) {
-              if (p.last_col != nullptr) static_cast<T*>(p.last_col)[irow[r]] = v;
-              if (p.rcol_out != nullptr) static_cast<T*>(p.rcol_out)[irow[r]] = v;
-            }
+          const G g = gcur[r][su];
+          O o;
+          T v = F::f(L, UL, U, UR, rc[r], cc, g, irow[r], c + p.col0, p.param_c, o);
+          if (CHECKED) {
+            // select-only fixups: boundary columns, virtual row; the right column is captured
+            // in registers (stored once per strip)
+            v = (c == -1) ? leftv[r] : v;
+            if (F::kMask & NB_UR) v = (c == n) ? rightv[r] : v;
+            if (vtop[r]) v = F::top(p, c + p.col0);
+            rlast[r] = (c == n - 1) ? v : rlast[r];
+            if (TABLE && rvalid[r] && (unsigned)c < (unsigned)n)
+              static_cast<O*>(p.table)[(int64_t)irow[r] * p.table_pitch + c] = o;
+          } else {
+            if (MODE == 1 && vtop[r]) v = F::top(p, c + p.col0);
+            if (TABLE && (MODE == 0 || rvalid[r]))
+              static_cast<O*>(p.table)[(int64_t)irow[r] * p.table_pitch + c] = o;
           }
+          nw[r] = v;
+          ncc[r] = cc;
+        }
+        bv[su] = nw[R - 1];
+        const T sv = (lane == 31) ? tv[su] : nw[R - 1];
+        const T rv = __shfl_sync(0xffffffffu, sv, (lane + 31) & 31);
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+#pragma unroll
+          for (int d = HV - 1; d > 0; --d) hist[r][d] = hist[r][d - 1];
+          hist[r][0] = nw[r];
+          if (SIG > 0) {
+#pragma unroll
+            for (int d = HC - 1; d > 0; --d) hcc[r][d] = hcc[r][d - 1];
+            hcc[r][0] = ncc[r];
+          }
+        }
+#pragma unroll
+        for (int d = FV - 1; d > 0; --d) fifo[d] = fifo[d - 1];
+        fifo[0] = rv;
+      }
+#pragma unroll
+      for (int su = 0; su < U; ++su) {
+        ccc[su] = ccn[su];
+#pragma unroll
+        for (int r = 0; r < R; ++r) gcur[r][su] = gnxt[r][su];
+      }
+      if (has_bot && lane == 31) {
+        if (U == 8) {
+          uint4* b4 = reinterpret_cast<uint4*>(bot + sb);
+          b4[0] = make_uint4(to_bits(bv[0]), to_bits(bv[1 % U]), to_bits(bv[2 % U]), to_bits(bv[3 % U]));
+          b4[1] = make_uint4(to_bits(bv[4 % U]), to_bits(bv[5 % U]), to_bits(bv[6 % U]), to_bits(bv[7 % U]));
         } else {
-          if (TABLE) static_cast<O*>(p.table)[irow[r] * p.table_pitch + c] = o;
-        }
-        nw[r] = v;
-        ncc[r] = cc;
-      }
-      // link I/O by lane 31 and the rotate-by-one shuffle
-      if (has_bot && lane == 31) bot[st] = Entry{nw[R - 1], ncc[R - 1]};
-      const Entry te = top[st];
-      const T sv = (lane == 31) ? te.v : nw[R - 1];
-      const CC scc = (lane == 31) ? te.cc : ncc[R - 1];
-      const int src = (lane + 31) & 31;
-      const T rv = __shfl_sync(0xffffffffu, sv, src);
-      const CC rcc = __shfl_sync(0xffffffffu, scc, src);
-      // shift histories
 #pragma unroll
-      for (int r = 0; r < R; ++r) {
-#pragma unroll
-        for (int d = HV - 1; d > 0; --d) hist[r][d] = hist[r][d - 1];
-        hist[r][0] = nw[r];
-        if (SIG > 0) {
-#pragma unroll
-          for (int d = HC - 1; d > 0; --d) hcc[r][d] = hcc[r][d - 1];
-          hcc[r][0] = ncc[r];
+          for (int su = 0; su < U; ++su) bot[sb + su] = bv[su];
         }
       }
-#pragma unroll
-      for (int d = FV - 1; d > 0; --d) fifo[d] = fifo[d - 1];
-      fifo[0] = rv;
-#pragma unroll
-      for (int d = FC - 1; d > 0; --d) fcc[d] = fcc[d - 1];
-      fcc[0] = rcc;
     }
   }
 };
+
+// Debug trace: stamp[0] = wait satisfied, stamp[1] = chunk done, per (strip, warp, chunk).
+__device__ __forceinline__ void trace_stamp(const FillParams& p, int s, int wid, int nwarps, int k,
+                                            int which) {
+  if (p.trace != nullptr && k < p.trace_chunks) {
+    const int64_t idx = (((int64_t)s * nwarps + wid) * p.trace_chunks + k) * 2 + which;
+    p.trace[idx] = globaltimer_ns();
+  }
+}
 
 template <class F, int R, int SIG, int E, int W, bool TABLE>
 __global__ void __launch_bounds__(Wave<F, R, SIG, E, W, TABLE>::kThreads)
@@ -198,7 +274,6 @@ wavefront_kernel(const FillParams p) {
   using WV = Wave<F, R, SIG, E, W, TABLE>;
   using T = typename WV::T;
   using CC = typename WV::CC;
-  using Entry = typename WV::Entry;
   constexpr int C = WV::C, NS = WV::NS, D = WV::D;
 
   __shared__ typename WV::Smem sm;
@@ -232,11 +307,27 @@ wavefront_kernel(const FillParams p) {
     if (wid < W) {
       // ------------------------------------------------------------------ compute warp
       WaveCompute<F, R, SIG, E, W, TABLE> cs;
+      cs.bring = sm.bring;
+      if (p.lcol_in != nullptr) {   // multi-GPU: rank g-1's right column of this strip
+        if (!wait_flag<true>(p.lflag_in + s, (p.wepoch << 32) | 1u, ctl, tmo)) return;
+      }
 #pragma unroll
       for (int r = 0; r < R; ++r) {
         const int64_t i = strip_top + (int64_t)(wid * 32 + lane) * R + r;
-        cs.irow[r] = i;
-        cs.rc[r] = (i >= 0 && i < p.rows) ? F::row_ctx(p, i) : typename WV::RC(0);
+        cs.irow[r] = (int)i;
+        cs.rvalid[r] = i >= 0 && i < p.rows;
+        cs.vtop[r] = i == -1;
+        cs.rc[r] = cs.rvalid[r] ? F::row_ctx(p, i) : typename WV::RC(0);
+        cs.rlast[r] = T(0);
+        if (cs.vtop[r]) {
+          cs.leftv[r] = F::top(p, p.col0 - 1);          // corner
+          cs.rightv[r] = F::top(p, p.col0 + n);
+        } else {
+          cs.leftv[r] = (p.lcol_in != nullptr && cs.rvalid[r])
+                            ? __ldcg(static_cast<const T*>(p.lcol_in) + i)
+                            : F::left(p, i);
+          cs.rightv[r] = F::right(p, i);
+        }
 #pragma unroll
         for (int d = 0; d < WV::HV; ++d) cs.hist[r][d] = T(0);
 #pragma unroll
@@ -244,11 +335,6 @@ wavefront_kernel(const FillParams p) {
       }
 #pragma unroll
       for (int d = 0; d < WV::FV; ++d) cs.fifo[d] = T(0);
-#pragma unroll
-      for (int d = 0; d < (WV::FC > 0 ? WV::FC : 1); ++d) cs.fcc[d] = CC(0);
-      if (p.lcol_in != nullptr) {   // multi-GPU: rank g-1's right column of this strip
-        if (!wait_flag<true>(p.lflag_in + s, (p.wepoch << 32) | 1u, ctl, tmo)) return;
-      }
       const bool virt = strip_top < 0;
       const int K = NQ + D;
       for (int k = 0; k < K; ++k) {
@@ -256,8 +342,8 @@ wavefront_kernel(const FillParams p) {
         const bool has_bot = k >= D;
         const uint32_t gt = iter * (uint32_t)NQ + (uint32_t)k;
         const uint32_t gb = iter * (uint32_t)NQ + (uint32_t)(k - D);
-        const Entry* top = sm.link[wid][0];
-        Entry* bot = sm.link[wid + 1][0];
+        const T* top = sm.link[wid][0];
+        T* bot = sm.link[wid + 1][0];
         if (has_top) {
           if (!mbar_wait(&sm.full[wid][gt % NS], (gt / NS) & 1u, ctl, tmo)) return;
           top = sm.link[wid][gt % NS];
@@ -268,71 +354,139 @@ wavefront_kernel(const FillParams p) {
           }
           bot = sm.link[wid + 1][gb % NS];
         }
+        if (lane == 0) trace_stamp(p, s, wid, W + 2, k, 0);
         const int tau_k = WV::TAU0 + k * C;
-        const bool steady = !virt && (tau_k - 31 * D - (R - 1) * SIG >= 0) && (tau_k + C < n);  // max column < n-1: last_col / rcol cells stay checked
-        if (steady)
-          cs.template chunk<false>(p, lane, tau_k, top, bot, has_bot);
+        // max column < n-1 keeps the last_col / rcol cells in the checked path
+        const bool steady = (tau_k - 31 * D - (R - 1) * SIG >= 0) && (tau_k + C < n);
+        if (steady && !virt)
+          cs.template chunk<0>(p, lane, tau_k, top, bot, has_bot);
+        else if (steady)
+          cs.template chunk<1>(p, lane, tau_k, top, bot, has_bot);
         else
-          cs.template chunk<true>(p, lane, tau_k, top, bot, has_bot);
+          cs.template chunk<2>(p, lane, tau_k, top, bot, has_bot);
         __syncwarp();
         if (lane == 0) {
           if (has_top) mbar_arrive(&sm.empty[wid][gt % NS]);
           if (has_bot) mbar_arrive(&sm.full[wid + 1][gb % NS]);
+          trace_stamp(p, s, wid, W + 2, k, 1);
+        }
+      }
+      // right column of every row of the strip: last_col output and/or rank g+1's window
+#pragma unroll
+      for (int r = 0; r < R; ++r) {
+        if (cs.rvalid[r]) {
+          if (p.last_col != nullptr) static_cast<T*>(p.last_col)[cs.irow[r]] = cs.rlast[r];
+          if (p.rcol_out != nullptr) static_cast<T*>(p.rcol_out)[cs.irow[r]] = cs.rlast[r];
         }
       }
       if (p.rcol_out != nullptr) __threadfence_system();
     } else if (wid == W) {
       // ------------------------------------------------------------------ loader warp
+      // Moves up to kBatch chunks per round trip: one flag check covers every chunk the
+      // previous strip has already published, and all their loads are in flight together.
       const T* prev = static_cast<const T*>(p.bnd) + (int64_t)(s - 1) * p.bnd_stride;
-      for (int k = 0; k < NQ; ++k) {
-        const uint32_t g = iter * (uint32_t)NQ + (uint32_t)k;
-        const int slot = g % NS;
-        if (g / NS >= 1) {
-          if (!mbar_wait(&sm.empty[0][slot], ((g / NS) - 1) & 1u, ctl, tmo)) return;
-        }
-        const int q = k * C + lane;
-        const int c = q - 32;
-        T v;
+      uint64_t avail = 0;   // chunks of strip s-1 known to be published
+      int k = 0;
+      while (k < NQ) {
+        int nb = min(kBatch, NQ - k);
         if (s > 0) {
-          if (!wait_flag<false>(p.prog + (s - 1), ep | (uint64_t)(k + 1), ctl, tmo)) return;
-          v = __ldcg(prev + q);
-        } else {
-          v = F::top(p, c + p.col0);
+          if ((uint64_t)(k + 1) > avail) {
+            uint64_t seen;
+            if (!wait_flag_relaxed(p.prog + (s - 1), ep | (uint64_t)(k + 1), ctl, tmo, seen)) return;
+            avail = seen - ep;
+          }
+          nb = min(nb, (int)(avail - (uint64_t)k));
         }
-        CC cc = (c >= 0 && c < n) ? F::col_ctx(p, c + p.col0) : CC(0);
-        sm.link[0][slot][lane] = Entry{v, cc};
-        __syncwarp();
-        if (lane == 0) mbar_arrive(&sm.full[0][slot]);
+        if (lane == 0) trace_stamp(p, s, wid, W + 2, k, 0);
+        T v[kBatch];
+        CC cc[kBatch];
+#pragma unroll
+        for (int j = 0; j < kBatch; ++j) {
+          const int q = (k + j) * C + lane;
+          const int c = q - 32;
+          if (j < nb) {
+            v[j] = (s > 0) ? __ldcg(prev + q) : F::top(p, c + p.col0);
+            cc[j] = (c >= 0 && c < n) ? F::col_ctx(p, c + p.col0) : CC(0);
+          }
+        }
+#pragma unroll
+        for (int j = 0; j < kBatch; ++j) {
+          if (j < nb) {
+            const uint32_t g = iter * (uint32_t)NQ + (uint32_t)(k + j);
+            const int slot = g % NS;
+            if (g / NS >= 1) {
+              if (!mbar_wait(&sm.empty[0][slot], ((g / NS) - 1) & 1u, ctl, tmo)) return;
+            }
+            sm.link[0][slot][lane] = v[j];
+            sm.bring[((k + j) * C + lane) & (kBRing - 1)] = cc[j];
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&sm.full[0][slot]);
+          }
+        }
+        if (lane == 0) trace_stamp(p, s, wid, W + 2, k, 1);
+        k += nb;
       }
     } else {
       // ------------------------------------------------------------------ storer warp
+      // Drains every chunk warp W-1 has already completed (up to kBatch) per round trip and
+      // publishes them with one release of the strip's progress flag.
       const bool last = (s == p.nstrips - 1);
       T* mine = static_cast<T*>(p.bnd) + (int64_t)s * p.bnd_stride;
       T rmin = T(0);
       bool have = false;
-      for (int k = 0; k < NQ; ++k) {
-        const uint32_t g = iter * (uint32_t)NQ + (uint32_t)k;
-        const int slot = g % NS;
-        if (!mbar_wait(&sm.full[W][slot], (g / NS) & 1u, ctl, tmo)) return;
-        const T v = sm.link[W][slot][lane].v;
-        __syncwarp();
-        if (lane == 0) mbar_arrive(&sm.empty[W][slot]);
-        const int q = k * C + lane;
-        const int c = q - 32;
-        if (!last) {
-          __stcg(mine + q, v);
-          __threadfence();
-          __syncwarp();
-          if (lane == 0) st_release_gpu(p.prog + s, ep | (uint64_t)(k + 1));
-        } else if (c >= 0 && c < n) {
-          if (p.last_row != nullptr) static_cast<T*>(p.last_row)[c] = v;
-          if (F::kScore == SCORE_LAST_CELL && c == n - 1 && p.score != nullptr && p.is_last_rank)
-            *static_cast<T*>(p.score) = v;
-          if (F::kScore == SCORE_ROW_MIN) {
-            rmin = have ? min(rmin, v) : v;
-            have = true;
+      int k = 0;
+      while (k < NQ) {
+        const uint32_t g0 = iter * (uint32_t)NQ + (uint32_t)k;
+        if (!mbar_wait(&sm.full[W][g0 % NS], (g0 / NS) & 1u, ctl, tmo)) return;
+        int nb = 1;
+        if (lane == 0) {
+          while (nb < kBatch && k + nb < NQ) {
+            const uint32_t g = g0 + (uint32_t)nb;
+            if (!mbar_try_wait(&sm.full[W][g % NS], (g / NS) & 1u)) break;
+            ++nb;
           }
         }
+        nb = __shfl_sync(0xffffffffu, nb, 0);
+        if (lane == 0) trace_stamp(p, s, wid, W + 2, k, 0);
+        T v[kBatch];
+#pragma unroll
+        for (int j = 0; j < kBatch; ++j) {
+          if (j < nb) {
+            const uint32_t g = g0 + (uint32_t)j;
+            if (j > 0) mbar_wait(&sm.full[W][g % NS], (g / NS) & 1u, ctl, tmo);   // already complete
+            v[j] = sm.link[W][g % NS][lane];
+          }
+        }
+        __syncwarp();
+        if (lane == 0) {
+#pragma unroll
+          for (int j = 0; j < kBatch; ++j)
+            if (j < nb) mbar_arrive(&sm.empty[W][(g0 + (uint32_t)j) % NS]);
+        }
+#pragma unroll
+        for (int j = 0; j < kBatch; ++j) {
+          if (j < nb) {
+            const int q = (k + j) * C + lane;
+            const int c = q - 32;
+            if (!last) {
+              __stcg(mine + q, v[j]);
+            } else if (c >= 0 && c < n) {
+              if (p.last_row != nullptr) static_cast<T*>(p.last_row)[c] = v[j];
+              if (F::kScore == SCORE_LAST_CELL && c == n - 1 && p.score != nullptr && p.is_last_rank)
+                *static_cast<T*>(p.score) = v[j];
+              if (F::kScore == SCORE_ROW_MIN) {
+                rmin = have ? min(rmin, v[j]) : v[j];
+                have = true;
+              }
+            }
+          }
+        }
+        if (!last) {
+          __syncwarp();   // orders every lane's stores before lane 0's (cumulative) release
+          if (lane == 0) st_release_gpu(p.prog + s, ep | (uint64_t)(k + nb));
+        }
+        if (lane == 0) trace_stamp(p, s, wid, W + 2, k, 1);
+        k += nb;
       }
       if (F::kScore == SCORE_ROW_MIN && last && p.score != nullptr) {
         for (int off = 16; off > 0; off >>= 1) {
