@@ -137,7 +137,7 @@ const VariantGeom* variant_geom(int id) {
   return nullptr;
 }
 constexpr int kWfWarps = 4;           // must match wavefront_launch.cuh
-constexpr int kPrevBandRows = 32;     // must match prevrow.cu
+constexpr int kPrevBandRows = 64;     // must match prevrow.cu
 constexpr int kPrevBW = 128;
 constexpr int kPrevRing = 4;
 constexpr int kPrevThreads = 256;
@@ -327,8 +327,20 @@ lddp_status launch(lddp_plan_t pl, const FillParams& p, cudaStream_t s) {
     e = (cudaError_t)r;
   } else if (pl->kind == 1) {
     const int64_t ntasks = (int64_t)pl->nblocks * pl->nbands;
+    FillParams q = p;
+    // TMA streaming path: 32-bit costs, W % 4 == 0, 16-byte aligned rows (lddp.h documents the
+    // fallback); block_cols = -1 selects it
+    const bool tma = (q.cols % 4 == 0) && (q.grid_pitch % 4 == 0) &&
+                     ((reinterpret_cast<uintptr_t>(q.grid) & 15) == 0) && env_int("LDDP_PREVROW_TMA", 1);
     int grid = (int)std::min<int64_t>(pl->grid, (ntasks + 7) / 8);
-    e = lddp::launch_prevrow(pl->desc.func, p, grid, s);
+    if (tma) {
+      // x2 CTAs of 4 warps; about two bands of tasks resident (more only spin on flags)
+      q.block_cols = -1;
+      const int64_t want = std::max<int64_t>(1, (2 * (int64_t)pl->nblocks + 7) / 8);
+      grid = (int)std::max<int64_t>(1, std::min<int64_t>({(int64_t)pl->grid / 2, (ntasks + 7) / 8, want}));
+      if (const char* g = getenv("LDDP_PREVROW_CTAS")) grid = std::max(1, atoi(g) / 2);
+    }
+    e = lddp::launch_prevrow(pl->desc.func, q, grid, s);
   } else {
     e = lddp::launch_invl(pl->desc.func, p, pl->grid, s);
   }
