@@ -41,6 +41,7 @@ struct CellLCS {
   __device__ static T left(const FillParams&, int64_t) { return 0; }
   __device__ static T right(const FillParams&, int64_t) { return 0; }
   __device__ static GridT load(const FillParams&, int64_t, int) { return 0; }
+  __device__ static void prefetch_l1(const FillParams&, int64_t, int) {}
   __device__ __forceinline__ static T f(T L, T UL, T U, T, RowCtx a, ColCtx b, GridT, int64_t,
                                         int, int, OutT& o) {
     T v = max(max(U, L), UL + (a == b ? 1 : 0));
@@ -71,6 +72,7 @@ struct CellLev {
   __device__ static T left(const FillParams&, int64_t i) { return (T)(i + 1); }   // f(i+1, 0)
   __device__ static T right(const FillParams&, int64_t) { return 0; }
   __device__ static GridT load(const FillParams&, int64_t, int) { return 0; }
+  __device__ static void prefetch_l1(const FillParams&, int64_t, int) {}
   __device__ __forceinline__ static T f(T L, T UL, T U, T, RowCtx a, ColCtx b, GridT, int64_t,
                                         int, int, OutT& o) {
     T v = (a == b) ? UL : 1 + min(min(U, L), UL);
@@ -102,6 +104,7 @@ struct CellDTW {
   __device__ static T left(const FillParams&, int64_t) { return __int_as_float(0x7f800000); }
   __device__ static T right(const FillParams&, int64_t) { return __int_as_float(0x7f800000); }
   __device__ static GridT load(const FillParams&, int64_t, int) { return 0.0f; }
+  __device__ static void prefetch_l1(const FillParams&, int64_t, int) {}
   __device__ __forceinline__ static T f(T L, T UL, T U, T, RowCtx x, ColCtx y, GridT, int64_t,
                                         int, int, OutT& o) {
     float cost = fabsf(__fsub_rn(x, y));
@@ -126,14 +129,19 @@ struct CellFS {
   using OutT = uint8_t;
   static constexpr uint32_t kMask = NB_L | NB_UL | NB_U | NB_UR;
   static constexpr bool kGridIn = true;
+  static constexpr bool kByteIO = true;   // uint8 grid in, uint8 table out (word-vectorisable)
   static constexpr int kScore = SCORE_NONE;
   __device__ static RowCtx row_ctx(const FillParams&, int64_t) { return 0; }
   __device__ static ColCtx col_ctx(const FillParams&, int) { return 0; }
+  __device__ static GridT from_byte(uint32_t b) { return (float)b; }
   __device__ static T top(const FillParams&, int) { return 0.0f; }
   __device__ static T left(const FillParams&, int64_t) { return 0.0f; }
   __device__ static T right(const FillParams&, int64_t) { return 0.0f; }
   __device__ static GridT load(const FillParams& p, int64_t i, int c) {
     return (float)__ldg(static_cast<const uint8_t*>(p.grid) + i * p.grid_pitch + c);
+  }
+  __device__ static void prefetch_l1(const FillParams& p, int64_t i, int c) {
+    asm volatile("prefetch.global.L1 [%0];" ::"l"(static_cast<const uint8_t*>(p.grid) + i * p.grid_pitch + c));
   }
   __device__ __forceinline__ static T f(T L, T UL, T U, T UR, RowCtx, ColCtx, GridT in, int64_t,
                                         int, int, OutT& o) {
@@ -170,6 +178,9 @@ struct CellMinPath3 {
   __device__ static GridT load(const FillParams& p, int64_t i, int c) {
     return __ldg(static_cast<const int32_t*>(p.grid) + i * p.grid_pitch + c);
   }
+  __device__ static void prefetch_l1(const FillParams& p, int64_t i, int c) {
+    asm volatile("prefetch.global.L1 [%0];" ::"l"(static_cast<const int32_t*>(p.grid) + i * p.grid_pitch + c));
+  }
   __device__ __forceinline__ static T f(T, T UL, T U, T UR, RowCtx, ColCtx, GridT g, int64_t,
                                         int, int, OutT& o) {
     T v = g + min(min(UL, U), UR);
@@ -198,6 +209,9 @@ struct CellMin2Plus {
   __device__ static GridT load(const FillParams& p, int64_t i, int c) {
     return __ldg(static_cast<const int32_t*>(p.grid) + i * p.grid_pitch + c);
   }
+  __device__ static void prefetch_l1(const FillParams& p, int64_t i, int c) {
+    asm volatile("prefetch.global.L1 [%0];" ::"l"(static_cast<const int32_t*>(p.grid) + i * p.grid_pitch + c));
+  }
   __device__ __forceinline__ static T f(T, T UL, T U, T, RowCtx, ColCtx, GridT g, int64_t i,
                                         int, int pc, OutT& o) {
     T v = (i == 0) ? g : min(UL, U) + pc;
@@ -225,6 +239,9 @@ struct CellDiagMaxPlus {
   __device__ static T right(const FillParams&, int64_t) { return 0; }
   __device__ static GridT load(const FillParams& p, int64_t i, int c) {
     return __ldg(static_cast<const int32_t*>(p.grid) + i * p.grid_pitch + c);
+  }
+  __device__ static void prefetch_l1(const FillParams& p, int64_t i, int c) {
+    asm volatile("prefetch.global.L1 [%0];" ::"l"(static_cast<const int32_t*>(p.grid) + i * p.grid_pitch + c));
   }
   __device__ __forceinline__ static T f(T, T UL, T, T, RowCtx, ColCtx, GridT g, int64_t i,
                                         int gc, int pc, OutT& o) {

@@ -36,6 +36,7 @@ constexpr int kChunk = 32;  // link chunk = 32 entries = one per lane
 constexpr int kUnroll = 8;  // steps per unrolled loop body
 constexpr int kBatch = 4;   // chunks moved per loader / storer round trip
 constexpr int kBRing = 4096; // column-context ring (entries); index = (column + 32) & (kBRing - 1)
+constexpr int kGridPrefetchCols = 256;  // L1 prefetch distance of grid rows (columns)
 
 
 template <class F, int R, int SIG, int E, int W, bool TABLE>
@@ -77,6 +78,11 @@ __device__ __forceinline__ bool cta_sync(uint64_t* bar, uint32_t& phase, Control
   return ok;
 }
 
+template <class F, class = void>
+struct ByteIO { static constexpr bool value = false; };
+template <class F>
+struct ByteIO<F, decltype(void(F::kByteIO))> { static constexpr bool value = F::kByteIO; };
+
 template <class T>
 __device__ __forceinline__ T bits_to(uint32_t x) {
   T t;
@@ -100,6 +106,9 @@ struct WaveCompute {
   using O = typename WV::O;
   static constexpr int C = WV::C, D = WV::D, HV = WV::HV, HC = WV::HC, FV = WV::FV;
   static_assert(sizeof(T) == 4, "link values are 32-bit");
+  // uint8 image in / out as aligned 32-bit words: every lane-row's column must share the step's
+  // residue mod 4 (R = 1 and D % 4 == 0), and chunk starts are multiples of 4.
+  static constexpr bool kVec = ByteIO<F>::value && R == 1 && (D % 4 == 0) && ((WV::TAU0 % 4) == 0);
 
   T hist[R][HV];   // hist[r][d] = value of row r at step tau-1-d
   CC hcc[R][HC];   // hcc[r][d]  = column context of row r at step tau-1-d (SIG > 0)
@@ -126,6 +135,20 @@ struct WaveCompute {
 #pragma unroll
       for (int r = 0; r < R; ++r) {
         const int c = c0 - r * SIG;
+        if constexpr (kVec) {
+          if (su % 4 == 0) {
+            // one aligned word covers this step and the next three (rows are padded to 4 B)
+            uint32_t w = 0;
+            const bool ok = rvalid[r] && c >= 0 && c < n;
+            if (MODE == 0 || ok)
+              w = __ldg(reinterpret_cast<const uint32_t*>(static_cast<const uint8_t*>(p.grid) +
+                                                          (int64_t)irow[r] * p.grid_pitch + c));
+#pragma unroll
+            for (int q = 0; q < 4; ++q)
+              if (su + q < U) g[r][su + q] = F::from_byte((w >> (8 * q)) & 0xffu);
+          }
+          continue;
+        }
         if (!F::kGridIn) {
           g[r][su] = G(0);
         } else if (MODE == 2) {
@@ -158,6 +181,15 @@ struct WaveCompute {
     // so the L1 / L2 latency of those loads is off the per-step critical path.
     CC ccc[U];
     G gcur[R][U];
+    if (F::kGridIn) {
+      // pull each lane-row's grid line 256 columns ahead into L1 (the per-cell loads of the
+      // next chunks then hit L1; an image row is streamed once per lane-row)
+#pragma unroll
+      for (int r = 0; r < R; ++r) {
+        const int c = tau_k - lane_off - r * SIG + kGridPrefetchCols;
+        if (rvalid[r] && c >= 0 && c < n) F::prefetch_l1(p, irow[r], c);
+      }
+    }
     prefetch<MODE, U>(p, lane_off, tau_k, ccc, gcur);
 #pragma unroll 1
     for (int sb = 0; sb < C; sb += U) {
@@ -175,6 +207,7 @@ struct WaveCompute {
         for (int su = 0; su < U; ++su) tv[su] = top[sb + su];
       }
       T bv[U];
+      uint32_t owd = 0;   // packed output bytes (kVec)
 #pragma unroll
       for (int su = 0; su < U; ++su) {
         const int tau = tau_k + sb + su;
@@ -215,8 +248,16 @@ struct WaveCompute {
               static_cast<O*>(p.table)[(int64_t)irow[r] * p.table_pitch + c] = o;
           } else {
             if (MODE == 1 && vtop[r]) v = F::top(p, c + p.col0);
-            if (TABLE && (MODE == 0 || rvalid[r]))
+            if constexpr (kVec && MODE == 0) {
+              // pack 4 output bytes, one aligned 32-bit store per 4 steps
+              const uint32_t ob = (uint32_t)o;
+              owd = (su % 4 == 0) ? ob : (owd | (ob << (8 * (su % 4))));
+              if (TABLE && su % 4 == 3)
+                *reinterpret_cast<uint32_t*>(static_cast<uint8_t*>(p.table) +
+                                             (int64_t)irow[r] * p.table_pitch + (c - 3)) = owd;
+            } else if (TABLE && (MODE == 0 || rvalid[r])) {
               static_cast<O*>(p.table)[(int64_t)irow[r] * p.table_pitch + c] = o;
+            }
           }
           nw[r] = v;
           ncc[r] = cc;
