@@ -129,7 +129,9 @@ int wf_dispatch(int func, int op, int variant, bool table, const FillParams* p, 
 // variant geometry: rows per lane R, intra-lane skew SIG, extra lag E
 struct VariantGeom { int id, R, SIG, E; };
 const VariantGeom kVariants[] = {
-    {0, 4, 0, 2}, {1, 4, 1, 1}, {2, 2, 1, 1}, {3, 8, 1, 1}, {10, 1, 2, 2}, {11, 2, 2, 2},
+    {0, 4, 0, 2}, {1, 4, 1, 1}, {2, 2, 1, 1}, {3, 8, 1, 1}, {4, 8, 0, 2}, {5, 4, 0, 1},
+    {6, 16, 0, 2}, {7, 8, 0, 3}, {8, 8, 1, 1}, {9, 8, 1, 1}, {12, 16, 1, 1}, {10, 1, 2, 2},
+    {11, 2, 2, 2},
 };
 const VariantGeom* variant_geom(int id) {
   for (const auto& v : kVariants)
@@ -443,7 +445,7 @@ lddp_status lddp_plan(const lddp_desc* desc, lddp_plan_t* out) {
         variant = (rows == 2) ? 11 : 10;
       } else {
         int v_env = env_int("LDDP_WF_VARIANT", -1);
-        if (v_env >= 0 && v_env < 10) variant = v_env;
+        if (v_env >= 0 && v_env != 10 && v_env != 11) variant = v_env;
         else if (rows == 2) variant = 2;
         else if (rows == 8) variant = 3;
         else variant = 0;

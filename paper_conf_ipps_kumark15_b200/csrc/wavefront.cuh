@@ -39,7 +39,7 @@ constexpr int kBRing = 4096; // column-context ring (entries); index = (column +
 constexpr int kGridPrefetchCols = 256;  // L1 prefetch distance of grid rows (columns)
 
 
-template <class F, int R, int SIG, int E, int W, bool TABLE>
+template <class F, int R, int SIG, int E, int W, bool TABLE, int GS = (SIG == 0 ? R : 1)>
 struct Wave {
   using T = typename F::T;
   using CC = typename F::ColCtx;
@@ -47,7 +47,8 @@ struct Wave {
   using G = typename F::GridT;
   using O = typename F::OutT;
   static constexpr int C = kChunk;
-  static constexpr int D = R * SIG + E;      // per-lane lag in steps
+  static constexpr int NG = R / GS;          // row groups per lane (rows chained within a group)
+  static constexpr int D = NG * SIG + E;     // per-lane lag in steps
   static constexpr int NS = 16;              // ring slots per link
   static constexpr int HV = SIG + 1;         // value history depth per row
   static constexpr int HC = SIG > 0 ? SIG : 1;  // column-context history depth per row
@@ -55,6 +56,8 @@ struct Wave {
   static constexpr int kThreads = (W + 2) * 32;
   static constexpr int TAU0 = -32 - SIG - E; // step at which lane 31 injects top entry q = 0
   static_assert(E >= 1, "need at least one step of shuffle slack");
+  static_assert(R % GS == 0, "row groups must tile the lane's rows");
+  static_assert(GS == 1 || SIG <= 1 || !(F::kMask & NB_UR), "UR needs every row skewed (GS = 1)");
   static_assert(SIG >= 2 || !(F::kMask & NB_UR), "UR needs the knight-move skew (SIG = 2)");
   static_assert(SIG + E >= 2 || !(F::kMask & NB_UR), "UR of row 0 must be at least one step old");
 
@@ -96,15 +99,15 @@ __device__ __forceinline__ uint32_t to_bits(T t) {
   return x;
 }
 
-template <class F, int R, int SIG, int E, int W, bool TABLE>
+template <class F, int R, int SIG, int E, int W, bool TABLE, int GS = (SIG == 0 ? R : 1)>
 struct WaveCompute {
-  using WV = Wave<F, R, SIG, E, W, TABLE>;
+  using WV = Wave<F, R, SIG, E, W, TABLE, GS>;
   using T = typename WV::T;
   using CC = typename WV::CC;
   using RC = typename WV::RC;
   using G = typename WV::G;
   using O = typename WV::O;
-  static constexpr int C = WV::C, D = WV::D, HV = WV::HV, HC = WV::HC, FV = WV::FV;
+  static constexpr int C = WV::C, D = WV::D, HV = WV::HV, HC = WV::HC, FV = WV::FV, NG = WV::NG;
   static_assert(sizeof(T) == 4, "link values are 32-bit");
   // uint8 image in / out as aligned 32-bit words: every lane-row's column must share the step's
   // residue mod 4 (R = 1 and D % 4 == 0), and chunk starts are multiples of 4.
@@ -134,7 +137,7 @@ struct WaveCompute {
       cc[su] = bring[(c0 + 32) & (kBRing - 1)];
 #pragma unroll
       for (int r = 0; r < R; ++r) {
-        const int c = c0 - r * SIG;
+        const int c = c0 - (r / GS) * SIG;
         if constexpr (kVec) {
           if (su % 4 == 0) {
             // one aligned word covers this step and the next three (rows are padded to 4 B)
@@ -186,7 +189,7 @@ struct WaveCompute {
       // next chunks then hit L1; an image row is streamed once per lane-row)
 #pragma unroll
       for (int r = 0; r < R; ++r) {
-        const int c = tau_k - lane_off - r * SIG + kGridPrefetchCols;
+        const int c = tau_k - lane_off - (r / GS) * SIG + kGridPrefetchCols;
         if (rvalid[r] && c >= 0 && c < n) F::prefetch_l1(p, irow[r], c);
       }
     }
@@ -215,7 +218,7 @@ struct WaveCompute {
         CC ncc[R];
 #pragma unroll
         for (int r = 0; r < R; ++r) {
-          const int c = tau - lane_off - r * SIG;
+          const int c = tau - lane_off - (r / GS) * SIG;
           T L = hist[r][0], U, UL, UR;
           CC cc;
           if (r == 0) {
@@ -223,14 +226,16 @@ struct WaveCompute {
             UL = fifo[SIG + E];
             UR = fifo[(SIG + E >= 2) ? SIG + E - 2 : 0];
             cc = ccc[su];
+          } else if (SIG == 0 || r % GS != 0) {
+            // inside a row group: the row above is at the same column this step
+            U = nw[r - 1];
+            cc = ncc[r - 1];
+            UL = hist[r - 1][0];
+            UR = U;   // unused (UR needs GS = 1)
           } else {
-            if (SIG == 0) {
-              U = nw[r - 1];
-              cc = ncc[0];
-            } else {
-              U = hist[r - 1][SIG > 0 ? SIG - 1 : 0];
-              cc = hcc[r - 1][SIG > 0 ? SIG - 1 : 0];
-            }
+            // first row of a skewed group: the row above is SIG steps ahead
+            U = hist[r - 1][SIG > 0 ? SIG - 1 : 0];
+            cc = hcc[r - 1][SIG > 0 ? SIG - 1 : 0];
             UL = hist[r - 1][SIG];
             UR = hist[r - 1][SIG >= 2 ? SIG - 2 : 0];
           }
@@ -309,10 +314,10 @@ __device__ __forceinline__ void trace_stamp(const FillParams& p, int s, int wid,
   }
 }
 
-template <class F, int R, int SIG, int E, int W, bool TABLE>
-__global__ void __launch_bounds__(Wave<F, R, SIG, E, W, TABLE>::kThreads)
+template <class F, int R, int SIG, int E, int W, bool TABLE, int GS = (SIG == 0 ? R : 1)>
+__global__ void __launch_bounds__(Wave<F, R, SIG, E, W, TABLE, GS>::kThreads)
 wavefront_kernel(const FillParams p) {
-  using WV = Wave<F, R, SIG, E, W, TABLE>;
+  using WV = Wave<F, R, SIG, E, W, TABLE, GS>;
   using T = typename WV::T;
   using CC = typename WV::CC;
   constexpr int C = WV::C, NS = WV::NS, D = WV::D;
@@ -347,7 +352,7 @@ wavefront_kernel(const FillParams p) {
 
     if (wid < W) {
       // ------------------------------------------------------------------ compute warp
-      WaveCompute<F, R, SIG, E, W, TABLE> cs;
+      WaveCompute<F, R, SIG, E, W, TABLE, GS> cs;
       cs.bring = sm.bring;
       if (p.lcol_in != nullptr) {   // multi-GPU: rank g-1's right column of this strip
         if (!wait_flag<true>(p.lflag_in + s, (p.wepoch << 32) | 1u, ctl, tmo)) return;
@@ -398,7 +403,7 @@ wavefront_kernel(const FillParams p) {
         if (lane == 0) trace_stamp(p, s, wid, W + 2, k, 0);
         const int tau_k = WV::TAU0 + k * C;
         // max column < n-1 keeps the last_col / rcol cells in the checked path
-        const bool steady = (tau_k - 31 * D - (R - 1) * SIG >= 0) && (tau_k + C < n);
+        const bool steady = (tau_k - 31 * D - ((R - 1) / GS) * SIG >= 0) && (tau_k + C < n);
         if (steady && !virt)
           cs.template chunk<0>(p, lane, tau_k, top, bot, has_bot);
         else if (steady)

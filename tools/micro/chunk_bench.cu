@@ -12,10 +12,13 @@ __global__ void bench(FillParams p, int chunks, long long* out) {
   using T = typename WC::T;
   __shared__ alignas(16) T top[32];
   __shared__ alignas(16) T bot[32];
+  __shared__ typename WC::CC bring[kBRing];
   const int lane = threadIdx.x & 31;
   top[lane] = T(0);
+  for (int i = lane; i < kBRing; i += 32) bring[i] = typename WC::CC(F::col_ctx(p, i % 1000));
   __syncwarp();
   WC cs;
+  cs.bring = bring;
   for (int r = 0; r < R; ++r) {
     cs.irow[r] = lane * R + r + (MODE == 1 ? -1 : 0);
     cs.rvalid[r] = cs.irow[r] >= 0;
@@ -23,6 +26,7 @@ __global__ void bench(FillParams p, int chunks, long long* out) {
     cs.rc[r] = F::row_ctx(p, cs.rvalid[r] ? cs.irow[r] : 0);
     cs.leftv[r] = T(0);
     cs.rightv[r] = T(0);
+    cs.rlast[r] = T(0);
     for (int d = 0; d < WC::HV; ++d) cs.hist[r][d] = T(0);
     for (int d = 0; d < WC::HC; ++d) cs.hcc[r][d] = typename WC::CC(0);
   }
