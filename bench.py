@@ -115,6 +115,11 @@ class ClockSampler:
                 "samples": len(win)}
 
 
+def _coll_dev(dev):
+    """Device for collective tensors: the GPU with NCCL, the CPU with a gloo test group."""
+    return torch.device("cpu") if os.environ.get("LDDP_BENCH_BACKEND", "nccl") != "nccl" else dev
+
+
 def dist_info():
     ws = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -200,7 +205,7 @@ def time_device(pb, lddp, steps, warmup, dev, world, flush):
     ms = [s.elapsed_time(e) for s, e in ev]
     total = sum(ms)
     if world > 1:
-        tt = torch.tensor([total], dtype=torch.float64, device=dev)
+        tt = torch.tensor([total], dtype=torch.float64, device=_coll_dev(dev))
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         total = float(tt.item())
     return total / steps, ms, t0, t1
@@ -248,7 +253,7 @@ def time_e2e(pb, lddp, steps, dev, world):
         res.copy_(pb["t"]["score"], non_blocking=True)
         torch.cuda.synchronize(dev)
     dt = (time.perf_counter() - t0) / steps
-    tt = torch.tensor([dt], dtype=torch.float64, device=dev)
+    tt = torch.tensor([dt], dtype=torch.float64, device=_coll_dev(dev))
     dist.all_reduce(tt, op=dist.ReduceOp.MAX)
     return float(tt.item()), pb["h2d"], 4
 
@@ -401,11 +406,20 @@ def main():
 
     from paper_conf_ipps_kumark15_b200 import lddp
 
+    # Test hooks (not used by the driver): LDDP_BENCH_SAME_DEVICE=1 puts every rank on cuda:0 and
+    # LDDP_BENCH_BACKEND=gloo uses a CPU process group -- exercises the cross-process CUDA-IPC
+    # window path on a single GPU (set LDDP_GRID_CTAS so all ranks' kernels are co-resident).
+    if os.environ.get("LDDP_BENCH_SAME_DEVICE") == "1":
+        local = 0
     dev = torch.device("cuda", local)
     torch.cuda.set_device(dev)
     if world > 1:
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=dev)
+        backend = os.environ.get("LDDP_BENCH_BACKEND", "nccl")
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group(backend)
     peaks = load_peaks()
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
     sampler = ClockSampler(local)
