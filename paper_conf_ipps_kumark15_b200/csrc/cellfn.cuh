@@ -141,7 +141,7 @@ struct CellFS {
     return (float)__ldg(static_cast<const uint8_t*>(p.grid) + i * p.grid_pitch + c);
   }
   __device__ static void prefetch_l1(const FillParams& p, int64_t i, int c) {
-    asm volatile("prefetch.global.L1 [%0];" ::"l"(static_cast<const uint8_t*>(p.grid) + i * p.grid_pitch + c));
+    asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(static_cast<const uint8_t*>(p.grid) + i * p.grid_pitch + c));
   }
   __device__ __forceinline__ static T f(T L, T UL, T U, T UR, RowCtx, ColCtx, GridT in, int64_t,
                                         int, int, OutT& o) {
@@ -179,7 +179,7 @@ struct CellMinPath3 {
     return __ldg(static_cast<const int32_t*>(p.grid) + i * p.grid_pitch + c);
   }
   __device__ static void prefetch_l1(const FillParams& p, int64_t i, int c) {
-    asm volatile("prefetch.global.L1 [%0];" ::"l"(static_cast<const int32_t*>(p.grid) + i * p.grid_pitch + c));
+    asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(static_cast<const int32_t*>(p.grid) + i * p.grid_pitch + c));
   }
   __device__ __forceinline__ static T f(T, T UL, T U, T UR, RowCtx, ColCtx, GridT g, int64_t,
                                         int, int, OutT& o) {
@@ -210,7 +210,7 @@ struct CellMin2Plus {
     return __ldg(static_cast<const int32_t*>(p.grid) + i * p.grid_pitch + c);
   }
   __device__ static void prefetch_l1(const FillParams& p, int64_t i, int c) {
-    asm volatile("prefetch.global.L1 [%0];" ::"l"(static_cast<const int32_t*>(p.grid) + i * p.grid_pitch + c));
+    asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(static_cast<const int32_t*>(p.grid) + i * p.grid_pitch + c));
   }
   __device__ __forceinline__ static T f(T, T UL, T U, T, RowCtx, ColCtx, GridT g, int64_t i,
                                         int, int pc, OutT& o) {
@@ -241,7 +241,7 @@ struct CellDiagMaxPlus {
     return __ldg(static_cast<const int32_t*>(p.grid) + i * p.grid_pitch + c);
   }
   __device__ static void prefetch_l1(const FillParams& p, int64_t i, int c) {
-    asm volatile("prefetch.global.L1 [%0];" ::"l"(static_cast<const int32_t*>(p.grid) + i * p.grid_pitch + c));
+    asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(static_cast<const int32_t*>(p.grid) + i * p.grid_pitch + c));
   }
   __device__ __forceinline__ static T f(T, T UL, T, T, RowCtx, ColCtx, GridT g, int64_t i,
                                         int gc, int pc, OutT& o) {

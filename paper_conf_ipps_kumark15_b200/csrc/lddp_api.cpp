@@ -131,7 +131,7 @@ struct VariantGeom { int id, R, SIG, E; };
 const VariantGeom kVariants[] = {
     {0, 4, 0, 2}, {1, 4, 1, 1}, {2, 2, 1, 1}, {3, 8, 1, 1}, {4, 8, 0, 2}, {5, 4, 0, 1},
     {6, 16, 0, 2}, {7, 8, 0, 3}, {8, 8, 1, 1}, {9, 8, 1, 1}, {12, 16, 1, 1}, {10, 1, 2, 2},
-    {11, 2, 2, 2},
+    {11, 2, 2, 2}, {13, 1, 2, 1},
 };
 const VariantGeom* variant_geom(int id) {
   for (const auto& v : kVariants)
@@ -442,7 +442,9 @@ lddp_status lddp_plan(const lddp_desc* desc, lddp_plan_t* out) {
       int rows = d.tile_rows > 0 ? d.tile_rows : env_int("LDDP_ROWS_PER_LANE", 0);
       int variant;
       if (knight) {
+        int v_env = env_int("LDDP_WF_VARIANT", -1);
         variant = (rows == 2) ? 11 : 10;
+        if (v_env == 10 || v_env == 11 || v_env == 13) variant = v_env;
       } else {
         int v_env = env_int("LDDP_WF_VARIANT", -1);
         if (v_env >= 0 && v_env != 10 && v_env != 11) variant = v_env;

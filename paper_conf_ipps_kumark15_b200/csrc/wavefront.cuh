@@ -39,6 +39,11 @@ constexpr int kBRing = 4096; // column-context ring (entries); index = (column +
 constexpr int kGridPrefetchCols = 256;  // L1 prefetch distance of grid rows (columns)
 
 
+template <class F, class = void>
+struct ByteIO { static constexpr bool value = false; };
+template <class F>
+struct ByteIO<F, decltype(void(F::kByteIO))> { static constexpr bool value = F::kByteIO; };
+
 template <class F, int R, int SIG, int E, int W, bool TABLE, int GS = (SIG == 0 ? R : 1)>
 struct Wave {
   using T = typename F::T;
@@ -65,7 +70,11 @@ struct Wave {
     alignas(16) T link[W + 1][NS][C];
     uint64_t full[W + 1][NS];
     uint64_t empty[W + 1][NS];
-    typename F::ColCtx bring[kBRing];   // column contexts staged by the loader
+    typename F::ColCtx bring[F::kGridIn ? 32 : kBRing];   // column contexts staged by the loader
+    // byte-image f's (FS): per compute warp, 3 chunks of 32 row segments x 32 bytes of input and
+    // one chunk of output, rows padded to 9 words (conflict-free lane-row reads)
+    uint32_t stg_in[ByteIO<F>::value ? W : 1][ByteIO<F>::value ? 3 * 32 * 9 : 1];
+    uint32_t stg_out[ByteIO<F>::value ? W : 1][ByteIO<F>::value ? 32 * 9 : 1];
     uint64_t bar;        // CTA barrier (abort-aware)
     int strip;
   };
@@ -80,11 +89,6 @@ __device__ __forceinline__ bool cta_sync(uint64_t* bar, uint32_t& phase, Control
   phase ^= 1u;
   return ok;
 }
-
-template <class F, class = void>
-struct ByteIO { static constexpr bool value = false; };
-template <class F>
-struct ByteIO<F, decltype(void(F::kByteIO))> { static constexpr bool value = F::kByteIO; };
 
 template <class T>
 __device__ __forceinline__ T bits_to(uint32_t x) {
@@ -123,6 +127,54 @@ struct WaveCompute {
   bool vtop[R];    // the lane-row is strip 0's virtual row -1 (holds the top initialisation)
   bool rvalid[R];  // 0 <= row < m
   T rlast[R];      // the row's value at column n-1 (captured in boundary chunks)
+  G gA[R][kUnroll], gB[R][kUnroll];   // grid prefetch pipeline (kGridIn f's)
+  uint32_t* stg_in;    // this warp's input staging [3][32][9] words (kVec)
+  uint32_t* stg_out;   // this warp's output staging [32][9] words (kVec)
+  int row_base;        // global row of lane 0's row 0
+  int carry_tau;   // chunk start whose first two sub-blocks gA / gB hold (else invalid)
+
+  // Byte-image staging (kVec: R = 1, D = 4): lane-row rho's 32 input bytes of the chunk that
+  // starts at step tau are the columns [tau - rho*D, tau - rho*D + 32) -- 8 aligned words.  The
+  // warp copies them cooperatively, 8 lanes per row segment (4 segments per instruction, so
+  // each instruction touches 4 lines instead of 32), with cp.async two chunks ahead.
+  __device__ __forceinline__ void stage_load(const FillParams& p, const int lane, const int tau) const {
+    const int n = p.cols;
+    const int k = (tau - WV::TAU0) / C;
+    const uint8_t* grid = static_cast<const uint8_t*>(p.grid);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+      const int rho = 4 * i + (lane >> 3);
+      const int j = lane & 7;
+      const int col = tau - rho * D + 4 * j;
+      const int row = row_base + rho;
+      const bool ok = row >= 0 && row < p.rows && col >= 0 && col < n;   // row padded to 4 B
+      cp_async_4(&stg_in[((k % 3) * 32 + rho) * 9 + j], ok ? grid + (int64_t)row * p.grid_pitch + col : grid,
+                 ok ? 4u : 0u);
+    }
+    cp_async_commit();
+  }
+  // Cooperative store of the chunk's output bytes (packed by their lane-rows in stg_out).
+  __device__ __forceinline__ void stage_store(const FillParams& p, const int lane, const int tau) const {
+    const int n = p.cols;
+    uint8_t* out = static_cast<uint8_t*>(p.table);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+      const int rho = 4 * i + (lane >> 3);
+      const int j = lane & 7;
+      const int col = tau - rho * D + 4 * j;
+      const int row = row_base + rho;
+      if (row < 0 || row >= p.rows) continue;
+      const uint32_t w = stg_out[rho * 9 + j];
+      uint8_t* rp = out + (int64_t)row * p.table_pitch;
+      if (col >= 0 && col + 3 < n) {
+        *reinterpret_cast<uint32_t*>(rp + col) = w;
+      } else if (col + 3 >= 0 && col < n) {
+#pragma unroll
+        for (int q = 0; q < 4; ++q)
+          if (col + q >= 0 && col + q < n) rp[col + q] = (uint8_t)(w >> (8 * q));
+      }
+    }
+  }
 
   // Loads for the 8 steps starting at tau0: row 0's column context and each row's grid input.
   const CC* bring;  // shared-memory column-context ring (staged by the loader warp)
@@ -134,21 +186,19 @@ struct WaveCompute {
 #pragma unroll
     for (int su = 0; su < U; ++su) {
       const int c0 = tau0 + su - lane_off;
-      cc[su] = bring[(c0 + 32) & (kBRing - 1)];
+      cc[su] = F::kGridIn ? CC(0) : bring[(c0 + 32) & (kBRing - 1)];
 #pragma unroll
       for (int r = 0; r < R; ++r) {
         const int c = c0 - (r / GS) * SIG;
         if constexpr (kVec) {
           if (su % 4 == 0) {
-            // one aligned word covers this step and the next three (rows are padded to 4 B)
-            uint32_t w = 0;
-            const bool ok = rvalid[r] && c >= 0 && c < n;
-            if (MODE == 0 || ok)
-              w = __ldg(reinterpret_cast<const uint32_t*>(static_cast<const uint8_t*>(p.grid) +
-                                                          (int64_t)irow[r] * p.grid_pitch + c));
+            // one staged word covers this step and the next three (see stage_load)
+            const int k = (tau0 - WV::TAU0) / C;            // chunk index of this sub-block
+            const int w = ((tau0 - WV::TAU0) % C + su) / 4;  // word within the lane-row segment
+            const uint32_t wd = stg_in[((k % 3) * 32 + lane_off / D) * 9 + w];
 #pragma unroll
             for (int q = 0; q < 4; ++q)
-              if (su + q < U) g[r][su + q] = F::from_byte((w >> (8 * q)) & 0xffu);
+              if (su + q < U) g[r][su + q] = F::from_byte((wd >> (8 * q)) & 0xffu);
           }
           continue;
         }
@@ -193,12 +243,40 @@ struct WaveCompute {
         if (rvalid[r] && c >= 0 && c < n) F::prefetch_l1(p, irow[r], c);
       }
     }
+    // Grid inputs (image / cost rows) stream from DRAM: they are kept two sub-blocks ahead in
+    // a register pipeline (gA, gB) that also carries across chunk boundaries; the loads are
+    // always bounds-guarded so a carried value is valid whatever the next chunk's mode.
+    // Column contexts come from the shared-memory ring one sub-block ahead.
+    constexpr bool kDeep = F::kGridIn && !kVec;
+    if constexpr (kVec) {
+      stage_load(p, lane, tau_k + 2 * C);   // two chunks ahead
+      cp_async_wait_group<2>();             // this chunk's segments have landed (own copies)
+      __syncwarp();                         // ... and every lane's copies are visible
+    }
+    if (kDeep) {
+      if (carry_tau != tau_k) {
+        prefetch<2, U>(p, lane_off, tau_k, ccc, gA);
+        prefetch<2, U>(p, lane_off, tau_k + U, ccc, gB);
+      }
+    }
     prefetch<MODE, U>(p, lane_off, tau_k, ccc, gcur);
 #pragma unroll 1
     for (int sb = 0; sb < C; sb += U) {
       CC ccn[U];
       G gnxt[R][U];
-      if (sb + U < C) prefetch<MODE, U>(p, lane_off, tau_k + sb + U, ccn, gnxt);
+      if (kDeep) {
+#pragma unroll
+        for (int su = 0; su < U; ++su)
+#pragma unroll
+          for (int r = 0; r < R; ++r) {
+            gcur[r][su] = gA[r][su];
+            gA[r][su] = gB[r][su];
+          }
+        prefetch<2, U>(p, lane_off, tau_k + sb + 2 * U, ccn, gB);
+        if (sb + U < C) prefetch<MODE, U>(p, lane_off, tau_k + sb + U, ccn, gnxt);
+      } else {
+        if (sb + U < C) prefetch<MODE, U>(p, lane_off, tau_k + sb + U, ccn, gnxt);
+      }
       T tv[U];
       if (U == 8) {
         const uint4 q0 = reinterpret_cast<const uint4*>(top + sb)[0];
@@ -249,17 +327,20 @@ struct WaveCompute {
             if (F::kMask & NB_UR) v = (c == n) ? rightv[r] : v;
             if (vtop[r]) v = F::top(p, c + p.col0);
             rlast[r] = (c == n - 1) ? v : rlast[r];
-            if (TABLE && rvalid[r] && (unsigned)c < (unsigned)n)
-              static_cast<O*>(p.table)[(int64_t)irow[r] * p.table_pitch + c] = o;
-          } else {
-            if (MODE == 1 && vtop[r]) v = F::top(p, c + p.col0);
-            if constexpr (kVec && MODE == 0) {
-              // pack 4 output bytes, one aligned 32-bit store per 4 steps
+            if constexpr (kVec) {
+              // packed into this lane-row's output segment; stored cooperatively per chunk
               const uint32_t ob = (uint32_t)o;
               owd = (su % 4 == 0) ? ob : (owd | (ob << (8 * (su % 4))));
-              if (TABLE && su % 4 == 3)
-                *reinterpret_cast<uint32_t*>(static_cast<uint8_t*>(p.table) +
-                                             (int64_t)irow[r] * p.table_pitch + (c - 3)) = owd;
+              if (su % 4 == 3) stg_out[lane * 9 + (sb + su) / 4] = owd;
+            } else if (TABLE && rvalid[r] && (unsigned)c < (unsigned)n) {
+              static_cast<O*>(p.table)[(int64_t)irow[r] * p.table_pitch + c] = o;
+            }
+          } else {
+            if (MODE == 1 && vtop[r]) v = F::top(p, c + p.col0);
+            if constexpr (kVec) {
+              const uint32_t ob = (uint32_t)o;
+              owd = (su % 4 == 0) ? ob : (owd | (ob << (8 * (su % 4))));
+              if (su % 4 == 3) stg_out[lane * 9 + (sb + su) / 4] = owd;
             } else if (TABLE && (MODE == 0 || rvalid[r])) {
               static_cast<O*>(p.table)[(int64_t)irow[r] * p.table_pitch + c] = o;
             }
@@ -288,8 +369,10 @@ struct WaveCompute {
 #pragma unroll
       for (int su = 0; su < U; ++su) {
         ccc[su] = ccn[su];
+        if (!kDeep) {
 #pragma unroll
-        for (int r = 0; r < R; ++r) gcur[r][su] = gnxt[r][su];
+          for (int r = 0; r < R; ++r) gcur[r][su] = gnxt[r][su];
+        }
       }
       if (has_bot && lane == 31) {
         if (U == 8) {
@@ -300,6 +383,14 @@ struct WaveCompute {
 #pragma unroll
           for (int su = 0; su < U; ++su) bot[sb + su] = bv[su];
         }
+      }
+    }
+    if (kDeep) carry_tau = tau_k + C;   // gA / gB now hold the next chunk's first two sub-blocks
+    if constexpr (kVec) {
+      if (TABLE) {
+        __syncwarp();
+        stage_store(p, lane, tau_k);
+        __syncwarp();
       }
     }
   }
@@ -354,6 +445,10 @@ wavefront_kernel(const FillParams p) {
       // ------------------------------------------------------------------ compute warp
       WaveCompute<F, R, SIG, E, W, TABLE, GS> cs;
       cs.bring = sm.bring;
+      cs.carry_tau = INT_MIN;
+      cs.stg_in = sm.stg_in[ByteIO<F>::value ? wid : 0];
+      cs.stg_out = sm.stg_out[ByteIO<F>::value ? wid : 0];
+      cs.row_base = (int)(strip_top + (int64_t)wid * 32 * R);
       if (p.lcol_in != nullptr) {   // multi-GPU: rank g-1's right column of this strip
         if (!wait_flag<true>(p.lflag_in + s, (p.wepoch << 32) | 1u, ctl, tmo)) return;
       }
@@ -383,6 +478,10 @@ wavefront_kernel(const FillParams p) {
       for (int d = 0; d < WV::FV; ++d) cs.fifo[d] = T(0);
       const bool virt = strip_top < 0;
       const int K = NQ + D;
+      if constexpr (WaveCompute<F, R, SIG, E, W, TABLE, GS>::kVec) {   // staging prologue
+        cs.stage_load(p, lane, WV::TAU0);
+        cs.stage_load(p, lane, WV::TAU0 + C);
+      }
       for (int k = 0; k < K; ++k) {
         const bool has_top = k < NQ;
         const bool has_bot = k >= D;
@@ -416,6 +515,10 @@ wavefront_kernel(const FillParams p) {
           if (has_bot) mbar_arrive(&sm.full[wid + 1][gb % NS]);
           trace_stamp(p, s, wid, W + 2, k, 1);
         }
+      }
+      if constexpr (WaveCompute<F, R, SIG, E, W, TABLE, GS>::kVec) {
+        cp_async_wait_group<0>();   // staging copies issued past the strip's end must land before the
+        __syncwarp();               // next strip's prologue reuses their slots
       }
       // right column of every row of the strip: last_col output and/or rank g+1's window
 #pragma unroll
@@ -464,7 +567,7 @@ wavefront_kernel(const FillParams p) {
               if (!mbar_wait(&sm.empty[0][slot], ((g / NS) - 1) & 1u, ctl, tmo)) return;
             }
             sm.link[0][slot][lane] = v[j];
-            sm.bring[((k + j) * C + lane) & (kBRing - 1)] = cc[j];
+            if (!F::kGridIn) sm.bring[((k + j) * C + lane) & (kBRing - 1)] = cc[j];
             __syncwarp();
             if (lane == 0) mbar_arrive(&sm.full[0][slot]);
           }

@@ -21,6 +21,7 @@ enum WfVariant : int {
   WF_A_R16_G4 = 12, // anti-diagonal: 16 rows / lane = 4 chained groups of 4, skewed 1, E = 1
   WF_K_R1 = 10,     // knight-move: 1 row / lane, skew 2, E = 2
   WF_K_R2 = 11,     // knight-move: 2 rows / lane, skew 2, E = 2
+  WF_K_R1_E1 = 13,  // knight-move: 1 row / lane, skew 2, E = 1 (D = 3)
 };
 constexpr int kWfWarps = 4;
 

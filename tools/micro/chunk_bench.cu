@@ -8,7 +8,7 @@ using namespace lddp;
 
 template <class F, int R, int SIG, int E, int MODE>
 __global__ void bench(FillParams p, int chunks, long long* out) {
-  using WC = WaveCompute<F, R, SIG, E, 4, false>;
+  using WC = WaveCompute<F, R, SIG, E, 4, F::kGridIn>;
   using T = typename WC::T;
   __shared__ alignas(16) T top[32];
   __shared__ alignas(16) T bot[32];
@@ -19,6 +19,7 @@ __global__ void bench(FillParams p, int chunks, long long* out) {
   __syncwarp();
   WC cs;
   cs.bring = bring;
+  cs.carry_tau = INT_MIN;
   for (int r = 0; r < R; ++r) {
     cs.irow[r] = lane * R + r + (MODE == 1 ? -1 : 0);
     cs.rvalid[r] = cs.irow[r] >= 0;
@@ -76,6 +77,26 @@ int main() {
   run<CellLCS, 4, 1, 1, 2>("LCS", p, d);
   run<CellLCS, 8, 1, 1, 0>("LCS", p, d);
   run<CellLCS, 2, 1, 1, 0>("LCS", p, d);
+  uint8_t* img;
+  cudaMalloc(&img, (size_t)4096 * 16384);
+  cudaMemset(img, 100, (size_t)4096 * 16384);
+  p.grid = img;
+  p.grid_pitch = 16384;
+  p.cols = 16000;
+  uint8_t* outimg;
+  cudaMalloc(&outimg, (size_t)4096 * 16384);
+  p.table = outimg;
+  p.table_pitch = 16384;
+  run<CellFS, 1, 2, 2, 0>("FS", p, d);
+  run<CellFS, 1, 2, 2, 2>("FS", p, d);
+  p.grid_pitch = 0;
+  run<CellFS, 1, 2, 2, 0>("FS-in0", p, d);
+  p.table_pitch = 0;
+  run<CellFS, 1, 2, 2, 0>("FS-io0", p, d);
+  p.grid_pitch = 16384;
+  run<CellFS, 1, 2, 2, 0>("FS-out0", p, d);
+  p.table_pitch = 16384;
+  p.cols = n - 4096;
   p.a = y;
   p.b = y;
   run<CellDTW, 4, 0, 2, 0>("DTW", p, d);
