@@ -22,6 +22,14 @@ enum ScoreKind { SCORE_NONE = 0, SCORE_LAST_CELL = 1, SCORE_ROW_MIN = 2 };
 // [L88] Fig. 1(c) contributing set {L,UL,U}; textbook recurrence (reading R1) in the exact
 // integer form max(U, L, UL + [a_i = b_j]) (equal to the textbook branch form because
 // adjacent LCS cells differ by at most 1).
+// Run-time 1 for integer adds the compiler must not fold into VIADD: VIADD issues on the ALU
+// pipe together with ISETP / VIMNMX3, IMAD on the FMA pipe (balances the two pipes).
+__device__ __forceinline__ int32_t imad_add1(int32_t x, int32_t one) {
+  int32_t r;
+  asm("mad.lo.s32 %0, %1, %2, %2;" : "=r"(r) : "r"(x), "r"(one));
+  return r;
+}
+
 struct CellLCS {
   using T = int32_t;
   using RowCtx = int32_t;
@@ -40,6 +48,10 @@ struct CellLCS {
   __device__ static T top(const FillParams&, int) { return 0; }
   __device__ static T left(const FillParams&, int64_t) { return 0; }
   __device__ static T right(const FillParams&, int64_t) { return 0; }
+  // virtual rows above row 0 (adiag.cuh): a character that matches nothing, boundary 0 -- f
+  // then regenerates the all-zero row 0 of the table by itself
+  __device__ static RowCtx vrow() { return -1; }
+  __device__ static T vbig() { return 0; }
   __device__ static GridT load(const FillParams&, int64_t, int) { return 0; }
   __device__ static void prefetch_l1(const FillParams&, int64_t, int) {}
   __device__ __forceinline__ static T f(T L, T UL, T U, T, RowCtx a, ColCtx b, GridT, int64_t,
@@ -47,6 +59,16 @@ struct CellLCS {
     T v = max(max(U, L), UL + (a == b ? 1 : 0));
     o = v;
     return v;
+  }
+  // The same cell for adiag.cuh, given eq = [a_i = b_j] from the per-lane match table (one
+  // shared-memory lookup + one R2P per step instead of one ISETP per cell): the +1 is a
+  // predicated IMAD on the FMA pipe (`one` is a run-time 1), the 3-way max one VIMNMX3.
+  static constexpr bool kMatchCells = true;
+  __device__ __forceinline__ static T fad(T, T, T, RowCtx, ColCtx, int32_t) { return T(0); }
+  __device__ __forceinline__ static T fadm(T L, T UL, T U, bool eq, int32_t one) {
+    const T ulp = imad_add1(UL, one);
+    const T t = eq ? ulp : UL;
+    return max(max(U, L), t);
   }
 };
 
@@ -71,6 +93,10 @@ struct CellLev {
   __device__ static T top(const FillParams&, int gc) { return gc + 1; }           // f(0, gc+1)
   __device__ static T left(const FillParams&, int64_t i) { return (T)(i + 1); }   // f(i+1, 0)
   __device__ static T right(const FillParams&, int64_t) { return 0; }
+  // virtual rows (adiag.cuh): never-matching character, boundary 2^30 above row -1, so that
+  // row -1 = 1 + L regenerates f(0, j) = j (values stay >= 2^30 above it)
+  __device__ static RowCtx vrow() { return -1; }
+  __device__ static T vbig() { return 1 << 30; }
   __device__ static GridT load(const FillParams&, int64_t, int) { return 0; }
   __device__ static void prefetch_l1(const FillParams&, int64_t, int) {}
   __device__ __forceinline__ static T f(T L, T UL, T U, T, RowCtx a, ColCtx b, GridT, int64_t,
@@ -78,6 +104,15 @@ struct CellLev {
     T v = (a == b) ? UL : 1 + min(min(U, L), UL);
     o = v;
     return v;
+  }
+  // adiag.cuh form (eq from the match table): the textbook min(U+1, L+1, UL+[a!=b]), equal in
+  // integers to the form above because adjacent edit-distance cells differ by at most 1 (and
+  // in the virtual rows above row 0 every value is >= 2^30, so row -1 is still L+1).
+  static constexpr bool kMatchCells = true;
+  __device__ __forceinline__ static T fad(T, T, T, RowCtx, ColCtx, int32_t) { return T(0); }
+  __device__ __forceinline__ static T fadm(T L, T UL, T U, bool eq, int32_t one) {
+    const T t = eq ? UL : imad_add1(UL, one);
+    return min(min(imad_add1(U, one), imad_add1(L, one)), t);
   }
 };
 
@@ -103,6 +138,9 @@ struct CellDTW {
   __device__ static T top(const FillParams&, int gc) { return gc == -1 ? 0.0f : __int_as_float(0x7f800000); }
   __device__ static T left(const FillParams&, int64_t) { return __int_as_float(0x7f800000); }
   __device__ static T right(const FillParams&, int64_t) { return __int_as_float(0x7f800000); }
+  // virtual rows (adiag.cuh): x = +inf makes every cost +inf, so row -1 = +inf for j >= 0
+  __device__ static RowCtx vrow() { return __int_as_float(0x7f800000); }
+  __device__ static T vbig() { return __int_as_float(0x7f800000); }
   __device__ static GridT load(const FillParams&, int64_t, int) { return 0.0f; }
   __device__ static void prefetch_l1(const FillParams&, int64_t, int) {}
   __device__ __forceinline__ static T f(T L, T UL, T U, T, RowCtx x, ColCtx y, GridT, int64_t,
@@ -111,6 +149,11 @@ struct CellDTW {
     float v = __fadd_rn(cost, fminf(fminf(U, L), UL));
     o = v;
     return v;
+  }
+  static constexpr bool kMatchCells = false;
+  __device__ __forceinline__ static T fadm(T, T, T, bool, int32_t) { return T(0); }
+  __device__ __forceinline__ static T fad(T L, T UL, T U, RowCtx x, ColCtx y, int32_t) {
+    return __fadd_rn(fabsf(__fsub_rn(x, y)), fminf(fminf(U, L), UL));
   }
 };
 

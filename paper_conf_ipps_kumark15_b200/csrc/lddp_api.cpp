@@ -31,6 +31,7 @@ int wf_dispatch_minpath3(int, int, bool, const FillParams*, int, cudaStream_t);
 int wf_dispatch_min2plus(int, int, bool, const FillParams*, int, cudaStream_t);
 int wf_dispatch_diagmaxplus(int, int, bool, const FillParams*, int, cudaStream_t);
 }  // namespace lddp
+#include "ad_table.inc"
 
 using lddp::FillParams;
 
@@ -126,6 +127,40 @@ int wf_dispatch(int func, int op, int variant, bool table, const FillParams* p, 
   }
 }
 
+// Compiled adiag geometries (tools/gen_adiag.py): f, rows per lane R, lane lag E, warps per CTA W.
+struct AdGeom {
+  int func, R, E, W;
+  cudaError_t (*launch)(const FillParams&, int, cudaStream_t);
+};
+const AdGeom kAdGeoms[] = {
+LDDP_AD_TABLE_ROWS
+};
+
+// Lane-systolic anti-diagonal geometry model, constants from the B200
+// microbenchmarks in tools/micro (ad_step2.cu, lat.cu).  One warp's step (R cells per lane)
+// costs t = max(chain / E, issue) + ~12 cycles: the chain is R dependent cell latencies plus
+// the rotate SHFL (~27) and SEL; issue is ~4.2 instructions per cell; W / 4 warps share an SM
+// sub-partition.  A fill takes about  waves x n x t  (every lane sweeps every column)  plus the
+// pipeline lag: each warp starts 32E + ~12 steps after the one above, each CTA ~40 more (L2).
+struct AdModel { double ipc, lat; };
+AdModel ad_model(int func) {
+  switch (func) {
+    case LDDP_F_DTW: return {4.0, 9.0};          // FADD, FMNMX3, FADD; chain FMNMX3 -> FADD
+    case LDDP_F_LEVENSHTEIN: return {4.6, 14.0}; // ISETP, VIMNMX3, IMAD, SEL; chain of three
+    default: return {4.2, 4.5};                  // LCS: ISETP, IMAD, IMAD.MOV, VIMNMX3; chain VIMNMX3
+  }
+}
+double ad_cost(int func, int R, int E, int W, int64_t m, int64_t n, int sms) {
+  const AdModel md = ad_model(func);
+  const double share = W / 4.0;   // warps per SM sub-partition
+  const double t = std::max((md.lat * R + 31.0) / E, share * md.ipc * R) + 12.0;
+  const int64_t warps = (m + 32 * R - 1) / (32 * R);
+  const int64_t cap = (int64_t)W * sms;
+  const int64_t waves = (warps + cap - 1) / cap;
+  const double lag = (double)warps * (32.0 * E + 12.0) + (double)((warps + W - 1) / W) * 40.0;
+  return ((double)waves * (double)n + lag) * t;
+}
+
 // variant geometry: rows per lane R, intra-lane skew SIG, extra lag E
 struct VariantGeom { int id, R, SIG, E; };
 const VariantGeom kVariants[] = {
@@ -157,7 +192,8 @@ struct lddp_plan_s {
   lddp_desc desc;
   int kind;          // 0 = wavefront (anti-diag / knight), 1 = prev-row, 2 = inverted-L
   int variant;       // wavefront variant id
-  int R, SIG, E;
+  int R, SIG, E, W;
+  cudaError_t (*ad_launch)(const FillParams&, int, cudaStream_t);   // adiag geometry (kind 3)
   int sms;
   int grid;
   int occupancy;
@@ -309,6 +345,8 @@ void fill_common(lddp_plan_t pl, const lddp_inputs* in, const lddp_outputs* out,
   p.block_cols = kPrevBW;
   p.halo = kPrevBandRows;
   p.nblocks = pl->nblocks;
+  p.debug = env_int("LDDP_DEBUG", 0);
+  p.one = 1;
   // debug trace buffer: LDDP_TRACE=<device pointer as decimal>:<chunks per row>
   if (const char* tr = getenv("LDDP_TRACE")) {
     unsigned long long ptr = 0;
@@ -327,6 +365,9 @@ lddp_status launch(lddp_plan_t pl, const FillParams& p, cudaStream_t s) {
     int r = wf_dispatch(pl->desc.func, 0, pl->variant, p.table != nullptr, &p, grid, s);
     if (r < 0) return fail(LDDP_ERR_UNSUPPORTED, "wavefront variant %d not compiled for f=%d", pl->variant, pl->desc.func);
     e = (cudaError_t)r;
+  } else if (pl->kind == 3) {
+    int grid = std::min(pl->grid, p.nstrips);
+    e = pl->ad_launch(p, grid, s);
   } else if (pl->kind == 1) {
     const int64_t ntasks = (int64_t)pl->nblocks * pl->nbands;
     FillParams q = p;
@@ -436,7 +477,42 @@ lddp_status lddp_plan(const lddp_desc* desc, lddp_plan_t* out) {
     DeviceGuard dg(dev);
     const bool table = (d.outputs & LDDP_OUT_TABLE) != 0;
 
-    if (d.category == LDDP_CAT_ANTI_DIAGONAL || d.category == LDDP_CAT_KNIGHT_MOVE) {
+    const char* kern_env = getenv("LDDP_KERNEL");
+    const bool force_wf = kern_env != nullptr && strcmp(kern_env, "wavefront") == 0;
+    if (d.category == LDDP_CAT_ANTI_DIAGONAL && seq_func(d.func) && !table && !force_wf) {
+      // lane-systolic anti-diagonal kernel (adiag.cuh)
+      pl->kind = 3;
+      int Rq = d.tile_rows > 0 ? d.tile_rows : env_int("LDDP_AD_R", 0);
+      int Eq = env_int("LDDP_AD_E", 0);
+      int Wq = d.tile_warps > 0 ? d.tile_warps : env_int("LDDP_AD_W", 0);
+      double best = 1e300;
+      pl->R = 0;
+      for (const auto& g : kAdGeoms) {
+        if (g.func != d.func) continue;
+        if (Eq > 0 && g.E != Eq) continue;
+        if (Wq > 0 && g.W != Wq) continue;
+        double c = ad_cost(d.func, g.R, g.E, g.W, d.rows, std::max<int64_t>(d.cols, 1), pl->sms);
+        if (Rq > 0) c += 1e200 * std::abs(g.R - Rq);   // nearest compiled R to the request
+        if (c < best) { best = c; pl->R = g.R; pl->E = g.E; pl->W = g.W; pl->ad_launch = g.launch; }
+      }
+      if (pl->R == 0) {
+        delete pl;
+        return fail(LDDP_ERR_UNSUPPORTED, "no compiled adiag geometry for f=%d (E=%d W=%d)", d.func, Eq, Wq);
+      }
+      pl->SIG = 0;
+      pl->variant = -1;
+      pl->occupancy = 1;
+      pl->strip_rows = (int64_t)pl->W * 32 * pl->R;
+      pl->nstrips = (int)((d.rows + pl->strip_rows - 1) / pl->strip_rows);
+      pl->row0 = d.rows - (int64_t)pl->nstrips * pl->strip_rows;
+      pl->nchunks = (int)((d.cols + 31) / 32);
+      pl->bnd_stride = (int64_t)std::max(pl->nchunks, 1) * 32;   // (value, tag) pairs per strip row
+      int g = d.grid_ctas > 0 ? d.grid_ctas : env_int("LDDP_GRID_CTAS", 0);
+      pl->grid = g > 0 ? g : pl->sms;
+      pl->off_prog = 64;
+      pl->off_bnd = 256;
+      pl->ws_bytes = pl->off_bnd + (size_t)std::max(pl->nstrips - 1, 1) * pl->bnd_stride * 8;
+    } else if (d.category == LDDP_CAT_ANTI_DIAGONAL || d.category == LDDP_CAT_KNIGHT_MOVE) {
       pl->kind = 0;
       const bool knight = d.category == LDDP_CAT_KNIGHT_MOVE;
       int rows = d.tile_rows > 0 ? d.tile_rows : env_int("LDDP_ROWS_PER_LANE", 0);
@@ -521,13 +597,13 @@ lddp_status lddp_plan_workspace_size(lddp_plan_t pl, size_t* bytes) {
 
 lddp_status lddp_plan_describe(lddp_plan_t pl, char* buf, size_t len) {
   if (pl == nullptr || buf == nullptr || len == 0) return fail(LDDP_ERR_INVALID_ARG, "NULL argument");
-  static const char* kinds[] = {"wavefront", "prevrow", "invl"};
+  static const char* kinds[] = {"wavefront", "prevrow", "invl", "adiag"};
   snprintf(buf, len,
            "{\"kernel\": \"%s\", \"variant\": %d, \"rows_per_lane\": %d, \"skew\": %d, \"extra_lag\": %d, "
            "\"warps\": %d, \"grid\": %d, \"sms\": %d, \"occupancy\": %d, \"strip_rows\": %lld, "
            "\"strips\": %d, \"chunks\": %d, \"blocks\": %d, \"bands\": %d, \"workspace_bytes\": %zu}",
            kinds[pl->kind], pl->variant, pl->R, pl->SIG, pl->E,
-           pl->kind == 0 ? kWfWarps + 2 : (pl->kind == 1 ? kPrevThreads / 32 : kInvlThreads / 32), pl->grid,
+           pl->kind == 0 ? kWfWarps + 2 : (pl->kind == 1 ? kPrevThreads / 32 : (pl->kind == 3 ? pl->W : kInvlThreads / 32)), pl->grid,
            pl->sms, pl->occupancy, (long long)pl->strip_rows, pl->nstrips, pl->nchunks, pl->nblocks, pl->nbands,
            pl->ws_bytes);
   return LDDP_OK;
@@ -649,7 +725,7 @@ lddp_status lddp_status_check(lddp_plan_t pl, void* ws, void* stream) {
 lddp_status lddp_comm_create(lddp_plan_t pl, int32_t nranks, int32_t rank, lddp_comm_t* out) {
   if (pl == nullptr || out == nullptr) return fail(LDDP_ERR_INVALID_ARG, "NULL argument");
   if (nranks < 1 || rank < 0 || rank >= nranks) return fail(LDDP_ERR_INVALID_ARG, "bad rank %d / %d", rank, nranks);
-  if (pl->kind != 0 || pl->desc.category != LDDP_CAT_ANTI_DIAGONAL)
+  if ((pl->kind != 0 && pl->kind != 3) || pl->desc.category != LDDP_CAT_ANTI_DIAGONAL)
     return fail(LDDP_ERR_UNSUPPORTED, "multi-GPU column strips: anti-diagonal category only in this build");
   if (pl->desc.cols < nranks) return fail(LDDP_ERR_SHAPE, "cols < nranks");
   DeviceGuard dg(pl->desc.device);
@@ -752,8 +828,13 @@ lddp_status lddp_fill_multi(lddp_plan_t pl, const lddp_inputs* in, const lddp_ou
     p.cols = (int32_t)(c1 - c0);
     p.col0 = (int32_t)c0;
     p.cols_total = (int32_t)n;
-    p.nchunks = (int)((p.cols + 33 + 31) / 32);
-    p.bnd_stride = (int64_t)p.nchunks * 32;
+    if (pl->kind == 3) {
+      p.nchunks = (int)((p.cols + 31) / 32);
+      p.bnd_stride = (int64_t)std::max(p.nchunks, 1) * 32;
+    } else {
+      p.nchunks = (int)((p.cols + 33 + 31) / 32);
+      p.bnd_stride = (int64_t)p.nchunks * 32;
+    }
     const bool last = c->rank == c->nranks - 1;
     p.is_last_rank = last ? 1 : 0;
     if (p.last_row) p.last_row = static_cast<char*>(p.last_row) + c0 * cell_bytes(d.func);

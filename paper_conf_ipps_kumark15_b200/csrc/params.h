@@ -50,6 +50,8 @@ struct FillParams {
   // debug trace (env LDDP_TRACE): globaltimer stamps per (strip, warp, chunk), or NULL
   uint64_t* trace;
   int32_t trace_chunks;     // chunks per (strip, warp) row of the trace
+  int32_t one;              // always 1 (a run-time constant the compiler cannot fold)
+  int32_t debug;            // env LDDP_DEBUG bits (development): 1 = adiag warps without handoffs
 };
 
 // Launch entry points (one per category family).  Return cudaError_t of the launch.

@@ -136,6 +136,29 @@ struct Watch {
   }
 };
 
+// Polling wait with an early back-off: a consumer warp spinning on shared / global memory
+// competes with the producer warps of its SM for the MIO / LSU pipes (SHFL, LDS), so after a
+// couple of failed polls it sleeps between polls.
+struct Backoff {
+  uint64_t t0;
+  uint32_t spins;
+  __device__ __forceinline__ Backoff() : t0(0), spins(0) {}
+  __device__ __forceinline__ bool tick(Control* ctl, uint64_t timeout_ns) {
+    ++spins;
+    if (spins >= 2) __nanosleep(spins < 256 ? 32 : 256);
+    if ((spins & 255) != 0) return true;
+    if (ld_volatile_u32(&ctl->abort)) return false;
+    uint64_t now = globaltimer_ns();
+    if (t0 == 0) { t0 = now; return true; }
+    if (now - t0 > timeout_ns) {
+      atomicCAS(&ctl->status, 0u, 8u /* LDDP_ERR_TIMEOUT */);
+      atomicExch(&ctl->abort, 1u);
+      return false;
+    }
+    return true;
+  }
+};
+
 // Wait until an epoch-tagged flag (epoch << 32 | count) reaches `target`.
 template <bool kSys>
 __device__ __forceinline__ bool wait_flag(const uint64_t* flag, uint64_t target, Control* ctl,

@@ -13,7 +13,8 @@ import ctypes
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "liblddp.so")
+# LDDP_LIB_PATH: development A/B builds (make LIB=... BUILD=... EXTRA=...); default the in-tree build
+LIB_PATH = os.environ.get("LDDP_LIB_PATH") or os.path.join(_HERE, "liblddp.so")
 if not os.path.exists(LIB_PATH):
     raise ImportError(
         f"liblddp.so not found at {LIB_PATH}: build it with `python -c 'import __graft_entry__ as g; g.build()'` "

@@ -1,0 +1,96 @@
+"""GPU parity of the lane-systolic anti-diagonal kernel (adiag.cuh) against the CPU oracle:
+every compiled (rows per lane R, lane lag E) geometry, shapes around the strip height
+(4 warps x 32 lanes x R rows, bottom-aligned with virtual rows above row 0) and the chunk width
+(32 columns), persistent grids smaller than the strip count (several strips per CTA), repeated
+fills on one workspace (epoch-tagged boundary pairs).  LCS / Levenshtein bit-exact; DTW
+bit-exact and <= 1e-5 relative (north star)."""
+import os
+import sys
+
+import numpy as np
+import pytest
+
+import oracle
+from gpu_util import run_gpu
+from paper_conf_ipps_kumark15_b200 import inputs
+
+pytestmark = pytest.mark.gpu
+
+sys.path.insert(0, os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "tools"))
+from gen_adiag import GEOMS as _GEN  # noqa: E402  (the compiled (R, E, W) geometries)
+
+GEOMS = {"lcs": _GEN["LCS"][1], "levenshtein": _GEN["LEVENSHTEIN"][1], "dtw": _GEN["DTW"][1]}
+
+
+def _inputs(func, seed, m, n):
+    if func == "dtw":
+        return inputs.gen_walks(seed, m, n)
+    return inputs.gen_strings(seed, m, n)
+
+
+def _ref(func, a, b):
+    return {"lcs": oracle.lcs, "levenshtein": oracle.levenshtein, "dtw": oracle.dtw}[func](a, b)
+
+
+def _check(func, got, ref):
+    for k in ("score", "last_row", "last_col"):
+        g, r = np.asarray(got[k]), np.asarray(getattr(ref, k))
+        if func == "dtw":
+            assert np.allclose(g, r, rtol=1e-5, atol=0), k
+            assert np.array_equal(g.astype(np.float32).view(np.int32), r.astype(np.float32).view(np.int32)), k
+        else:
+            np.testing.assert_array_equal(g, r, err_msg=k)
+
+
+def _run(func, R, E, W, a, b, **kw):
+    old = {k: os.environ.get(k) for k in ("LDDP_AD_E", "LDDP_AD_W")}
+    os.environ["LDDP_AD_E"] = str(E)
+    os.environ["LDDP_AD_W"] = str(W)
+    try:
+        got = run_gpu(func, "anti_diagonal", a=a, b=b, outputs=("score", "last_row", "last_col"),
+                      tile_rows=R, **kw)
+    finally:
+        for k, v in old.items():
+            if v is None:
+                os.environ.pop(k, None)
+            else:
+                os.environ[k] = v
+    plan = got["plan"]
+    assert '"adiag"' in plan and f'"rows_per_lane": {R},' in plan and f'"extra_lag": {E},' in plan, plan
+    assert f'"warps": {W},' in plan, plan
+    return got
+
+
+def _cases():
+    for func, geoms in GEOMS.items():
+        for R, E, W in geoms:
+            sh = 32 * W * R
+            for m, n in [(1, 1), (1, 70), (70, 1), (sh - 1, 33), (sh, 32), (sh + 1, 31), (2 * sh + 5, 41),
+                         (3 * sh - 7, 72), (sh // 2 + 3, 1000), (997, 1009)]:
+                yield func, R, E, W, m, n
+
+
+@pytest.mark.parametrize("func,R,E,W,m,n", list(_cases()))
+def test_adiag_geometry(func, R, E, W, m, n):
+    a, b = _inputs(func, 31 * m + n + R, m, n)
+    _check(func, _run(func, R, E, W, a, b), _ref(func, a, b))
+
+
+@pytest.mark.parametrize("func", ["lcs", "levenshtein", "dtw"])
+@pytest.mark.parametrize("grid", [1, 2, 3])
+def test_adiag_small_grid(func, grid):
+    """More strips than CTAs: each CTA runs several strips in claim order (deadlock-free)."""
+    R, E, W = GEOMS[func][0]
+    m, n = 32 * W * R * 5 + 17, 300
+    a, b = _inputs(func, 5 + grid, m, n)
+    _check(func, _run(func, R, E, W, a, b, grid_ctas=grid, reps=3), _ref(func, a, b))
+
+
+@pytest.mark.parametrize("func", ["lcs", "levenshtein", "dtw"])
+def test_adiag_large(func):
+    """A few thousand rows and columns with the planner's own geometry choice."""
+    m, n = 6001, 5003
+    a, b = _inputs(func, 77, m, n)
+    got = run_gpu(func, "anti_diagonal", a=a, b=b, outputs=("score", "last_row", "last_col"), reps=2)
+    assert '"adiag"' in got["plan"]
+    _check(func, got, _ref(func, a, b))
