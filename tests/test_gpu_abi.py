@@ -110,7 +110,17 @@ def test_plan_describe_and_workspace(L):
     try:
         import json
         info = json.loads(L.lddp_plan_describe(plan))
-        assert info["kernel"] == "wavefront" and info["strips"] >= 1
+        # sequence f's without TABLE output run the lane-systolic adiag kernel
+        assert info["kernel"] == "adiag" and info["strips"] >= 1
+        assert info["strip_rows"] == 32 * info["warps"] * info["rows_per_lane"]
         assert L.lddp_plan_workspace_size(plan) > 0
+    finally:
+        L.lddp_plan_destroy(plan)
+    d = L.lddp_desc(rows=500, cols=300, category=L.CAT_ANTI_DIAGONAL, func=L.F_LCS,
+                    outputs=L.OUT_SCORE | L.OUT_TABLE)
+    plan = L.lddp_plan(d)
+    try:
+        import json
+        assert json.loads(L.lddp_plan_describe(plan))["kernel"] == "wavefront"   # TABLE output
     finally:
         L.lddp_plan_destroy(plan)

@@ -70,6 +70,23 @@ def test_seq_variants_antidiag(func, rows, shape):
 
 
 @pytest.mark.parametrize("func", ["lcs", "levenshtein", "dtw"])
+@pytest.mark.parametrize("rows", AD_VARIANTS)
+@pytest.mark.parametrize("shape", [(3, 5), (513, 95), (997, 1009), (2100, 1700)])
+def test_seq_variants_wavefront_kernel(func, rows, shape, monkeypatch):
+    """The strip-wavefront kernel (default for TABLE outputs) on score / last-row / last-column."""
+    monkeypatch.setenv("LDDP_KERNEL", "wavefront")
+    m, n = shape
+    a, b = _seq_inputs(func, 11 * m + n + rows, m, n)
+    ref = _oracle_seq(func, a, b)
+    got = run_gpu(func, "anti_diagonal", a=a, b=b, outputs=("score", "last_row", "last_col"),
+                  tile_rows=rows)
+    assert '"wavefront"' in got["plan"]
+    _assert_close(func, got["last_row"], ref.last_row)
+    _assert_close(func, got["last_col"], ref.last_col)
+    _assert_close(func, got["score"], ref.score)
+
+
+@pytest.mark.parametrize("func", ["lcs", "levenshtein", "dtw"])
 @pytest.mark.parametrize("rows", KN_VARIANTS)
 @pytest.mark.parametrize("shape", [(1, 1), (5, 2), (300, 257), (1025, 999)])
 def test_seq_under_knight_schedule(func, rows, shape):
