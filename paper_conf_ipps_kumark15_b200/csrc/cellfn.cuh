@@ -226,7 +226,7 @@ struct CellMinPath3 {
   }
   __device__ __forceinline__ static T f(T, T UL, T U, T UR, RowCtx, ColCtx, GridT g, int64_t,
                                         int, int, OutT& o) {
-    T v = g + min(min(UL, U), UR);
+    T v = g + __vimin3_s32(UL, U, UR);   // VIMNMX3
     o = v;
     return v;
   }

@@ -206,6 +206,9 @@ struct lddp_plan_s {
   // prev-row geometry
   int nblocks;
   int nbands;
+  int cb_variant;    // column-block persistent kernel (prevrow_cb.cu): -1 = not usable
+  int cb_nw;         // warps per CTA
+  int cb_nblocks;    // column blocks (one warp each)
   // workspace layout (bytes)
   size_t off_prog, off_bnd, ws_bytes;
   // own workspace + host-fill staging
@@ -368,6 +371,12 @@ lddp_status launch(lddp_plan_t pl, const FillParams& p, cudaStream_t s) {
   } else if (pl->kind == 3) {
     int grid = std::min(pl->grid, p.nstrips);
     e = pl->ad_launch(p, grid, s);
+  } else if (pl->kind == 1 && pl->cb_variant >= 0 && (p.grid_pitch % 4 == 0) &&
+             ((reinterpret_cast<uintptr_t>(p.grid) & 15) == 0)) {
+    FillParams q = p;
+    q.nblocks = pl->cb_nblocks;
+    int dummy[2];
+    e = lddp::launch_prevrow_cb(pl->desc.func, pl->cb_variant, q, pl->cb_nw, false, dummy, s);
   } else if (pl->kind == 1) {
     const int64_t ntasks = (int64_t)pl->nblocks * pl->nbands;
     FillParams q = p;
@@ -562,6 +571,31 @@ lddp_status lddp_plan(const lddp_desc* desc, lddp_plan_t* out) {
       pl->off_prog = 64;
       pl->off_bnd = align_up(pl->off_prog + (size_t)std::max(pl->nblocks, 1) * 16, 256);
       pl->ws_bytes = pl->off_bnd + (size_t)kPrevRing * pl->bnd_stride * cell_bytes(d.func);
+      // Column-block persistent kernel: every block co-resident (cooperative launch), W % 4 == 0
+      // (16-byte cost segments; the row pitch / base alignment is checked per fill).
+      pl->cb_variant = -1;
+      const int cbv = env_int("LDDP_CB_VARIANT", 5);
+      const int cbnw = std::max(1, std::min(8, env_int("LDDP_CB_WARPS", 2)));
+      if (cbv >= 0 && d.cols > 0 && d.rows > 0 && d.cols % 4 == 0) {
+        int q[2] = {0, 0};
+        FillParams dummy{};
+        if (lddp::launch_prevrow_cb(d.func, cbv, dummy, cbnw, true, q, nullptr) == cudaSuccess && q[0] > 0) {
+          const int64_t nbq = (d.cols + q[0] - 1) / q[0];
+          const int64_t ctas = (nbq + cbnw - 1) / cbnw;
+          if (q[1] > 0 && ctas <= (int64_t)q[1] * pl->sms) {
+            pl->cb_variant = cbv;
+            pl->cb_nw = cbnw;
+            pl->cb_nblocks = (int)nbq;
+            // workspace: row minima (4 B per block) + edge pairs [nb][4][2][HB <= 64] x 8 B
+            const size_t prog = align_up(64 + (size_t)nbq * 4, 256);
+            pl->off_prog = 64;
+            pl->off_bnd = std::max(pl->off_bnd, prog);
+            pl->ws_bytes = std::max(pl->ws_bytes, pl->off_bnd + (size_t)nbq * 4 * 2 * 64 * 8);
+          }
+        } else {
+          cudaGetLastError();
+        }
+      }
     } else {
       pl->kind = 2;
       const int64_t nd = d.rows + d.cols - 1;
@@ -598,14 +632,17 @@ lddp_status lddp_plan_workspace_size(lddp_plan_t pl, size_t* bytes) {
 lddp_status lddp_plan_describe(lddp_plan_t pl, char* buf, size_t len) {
   if (pl == nullptr || buf == nullptr || len == 0) return fail(LDDP_ERR_INVALID_ARG, "NULL argument");
   static const char* kinds[] = {"wavefront", "prevrow", "invl", "adiag"};
+  const bool cb = pl->kind == 1 && pl->cb_variant >= 0;
   snprintf(buf, len,
            "{\"kernel\": \"%s\", \"variant\": %d, \"rows_per_lane\": %d, \"skew\": %d, \"extra_lag\": %d, "
            "\"warps\": %d, \"grid\": %d, \"sms\": %d, \"occupancy\": %d, \"strip_rows\": %lld, "
            "\"strips\": %d, \"chunks\": %d, \"blocks\": %d, \"bands\": %d, \"workspace_bytes\": %zu}",
-           kinds[pl->kind], pl->variant, pl->R, pl->SIG, pl->E,
-           pl->kind == 0 ? kWfWarps + 2 : (pl->kind == 1 ? kPrevThreads / 32 : (pl->kind == 3 ? pl->W : kInvlThreads / 32)), pl->grid,
-           pl->sms, pl->occupancy, (long long)pl->strip_rows, pl->nstrips, pl->nchunks, pl->nblocks, pl->nbands,
-           pl->ws_bytes);
+           cb ? "prevrow_cb" : kinds[pl->kind], cb ? pl->cb_variant : pl->variant, pl->R, pl->SIG, pl->E,
+           cb ? pl->cb_nw
+              : (pl->kind == 0 ? kWfWarps + 2 : (pl->kind == 1 ? kPrevThreads / 32 : (pl->kind == 3 ? pl->W : kInvlThreads / 32))),
+           cb ? (pl->cb_nblocks + pl->cb_nw - 1) / pl->cb_nw : pl->grid,
+           pl->sms, cb ? 1 : pl->occupancy, (long long)pl->strip_rows, pl->nstrips, pl->nchunks,
+           cb ? pl->cb_nblocks : pl->nblocks, pl->nbands, pl->ws_bytes);
   return LDDP_OK;
 }
 

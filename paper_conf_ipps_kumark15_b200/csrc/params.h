@@ -58,6 +58,10 @@ struct FillParams {
 cudaError_t launch_wavefront(int func, int category, const FillParams& p, int rows_per_lane,
                              int warps, int grid, cudaStream_t stream);
 cudaError_t launch_prevrow(int func, const FillParams& p, int grid, cudaStream_t stream);
+// Column-block persistent prev-row kernel (cooperative launch).  query: out[0] = own columns
+// per warp, out[1] = co-resident CTAs per SM (nothing launched).
+cudaError_t launch_prevrow_cb(int func, int variant, const FillParams& p, int nw, bool query, int* out,
+                              cudaStream_t stream);
 cudaError_t launch_invl(int func, const FillParams& p, int grid, cudaStream_t stream);
 
 // Per-kernel occupancy query (blocks per SM) for the chosen configuration.

@@ -1,0 +1,329 @@
+// prevrow_cb.cu -- previous-row-only ("Horizontal", t = i) category, column-block persistent
+// kernel [L180-L195], Fig. 2(b).  The default prev-row kernel when the grid is 32-bit, W % 4 == 0
+// and the column blocks fit co-resident (cooperative launch); prevrow.cu is the fallback.
+//
+// Every cell of row i depends only on row i-1 (contributing set within {UL, U, UR}), so the
+// degree of parallelism is the row width in every iteration [L184].  The paper launches one
+// kernel per row [L184], [L251]; here ONE cooperative launch fills the whole table:
+//
+//  * Warp q owns the column block [q*BW, (q+1)*BW) for ALL rows: its DP state never leaves the
+//    register file.  Lane l holds VP consecutive columns of the extended window
+//    [q*BW - HB, (q+1)*BW + HB), EXT = 32*VP = BW + 2*HB.
+//  * Bands of HB rows.  Within a band the warp recomputes the two HB-column halos itself (the
+//    TRAPEZOID: garbage entering from the window's outer edges advances one column per row, so
+//    after HB rows it has not reached the block's own columns).  At each band boundary the warp
+//    publishes the HB own columns at each edge and replaces its halos with the neighbours'
+//    published edges: case-2 two-way halo of Table II [L265-L274], ([L193-L195]), one exchange
+//    per HB rows instead of one per row.
+//  * Edge exchange = (value, tag) 64-bit pairs in global memory (single-copy atomic): the
+//    consumer polls the data itself, no flag, no fence.  Tag = hash(fill epoch) + band.
+//  * Cost rows (the HBM stream, 4 B/cell) flow through a per-warp D-row shared-memory ring
+//    filled by 16-byte cp.async (LDGSTS.128, L1 bypass), D-1 rows ahead of the row being
+//    computed; every lane copies exactly the columns it later reads, so the ring needs no warp
+//    synchronisation at all.
+//  * The last band writes last_row and the row minimum (score).
+#include <cstdint>
+#include <climits>
+#include "cellfn.cuh"
+#include "params.h"
+#include "sync.cuh"
+
+namespace lddp {
+
+__device__ __forceinline__ void cb_cp16(void* dst, const void* src, uint32_t src_bytes) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(smem_u32(dst)), "l"(src), "r"(src_bytes)
+               : "memory");
+}
+__device__ __forceinline__ void cb_cp16s(uint32_t dst, const void* src, uint32_t src_bytes) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src), "r"(src_bytes) : "memory");
+}
+__device__ __forceinline__ void cb_st_pair2(uint64_t* p, uint64_t a, uint64_t b) {
+  asm volatile("st.relaxed.gpu.global.v2.u64 [%0], {%1, %2};" ::"l"(p), "l"(a), "l"(b) : "memory");
+}
+__device__ __forceinline__ void cb_ld_pair2(const uint64_t* p, uint64_t& a, uint64_t& b) {
+  asm volatile("ld.relaxed.gpu.global.v2.u64 {%0, %1}, [%2];" : "=l"(a), "=l"(b) : "l"(p) : "memory");
+}
+
+// One band of nr <= HB rows.  OUT: this lane holds out-of-table columns (their value is f's
+// boundary value in every row: one extra select per cell, taken only by the two edge blocks'
+// edge lanes -- warp-uniform for every other warp).
+template <class F, int VP, int D, bool TABLE, bool OUT>
+__device__ __forceinline__ void cb_band(const FillParams& p, typename F::T (&cur)[VP], typename F::GridT (&g)[VP],
+                                        const int nr, const int64_t r0,
+                                        const typename F::GridT* ring, int& cslot, uint32_t& idst, int& ileft,
+                                        const typename F::GridT* (&src)[VP / 4], const uint32_t (&ssz)[VP / 4],
+                                        const typename F::T (&outv)[VP], const uint32_t omask, const int e0,
+                                        const int j0, const int BW) {
+  using T = typename F::T;
+  using G = typename F::GridT;
+  constexpr int EXT = 32 * VP;
+  const int64_t pitch = p.grid_pitch;
+  const uint32_t ibeg = smem_u32(ring), iend = ibeg + (D - 1) * EXT * 4;
+#pragma unroll 2
+  for (int r = 0; r < nr; ++r) {
+    // issue row + D - 1 into the slot consumed last (32-bit shared address, wraps at the ring end)
+    if (ileft > 0) {
+#pragma unroll
+      for (int s = 0; s < VP / 4; ++s) {
+        cb_cp16s(idst + 16 * s, src[s], ssz[s]);
+        src[s] += pitch;
+      }
+    }
+    --ileft;
+    idst = (idst == iend) ? ibeg : idst + EXT * 4;
+    cp_async_commit();
+    cp_async_wait_group<D - 2>();    // the NEXT row's group has landed: load it now, use it next row
+    G gn[VP];
+    cslot = (cslot + 1 == D) ? 0 : cslot + 1;
+    const G* gs = ring + cslot * EXT;
+#pragma unroll
+    for (int s = 0; s < VP / 4; ++s) {
+      const int4 t = *reinterpret_cast<const int4*>(gs + 4 * s);
+      gn[4 * s] = t.x; gn[4 * s + 1] = t.y; gn[4 * s + 2] = t.z; gn[4 * s + 3] = t.w;
+    }
+    const int64_t row = r0 + r;
+    const T lv = __shfl_up_sync(0xffffffffu, cur[VP - 1], 1);   // lane 0: own value (halo garbage)
+    const T rv = __shfl_down_sync(0xffffffffu, cur[0], 1);
+    T nw_[VP];
+#pragma unroll
+    for (int v = 0; v < VP; ++v) {
+      const T UL = (v > 0) ? cur[v - 1] : lv;
+      const T U = cur[v];
+      const T UR = (v < VP - 1) ? cur[v + 1] : rv;
+      typename F::OutT o;
+      T x = F::f(U, UL, U, UR, typename F::RowCtx(0), typename F::ColCtx(0), g[v], row, e0 + v, p.param_c, o);
+      if (OUT) x = ((omask >> v) & 1u) ? outv[v] : x;
+      nw_[v] = x;
+      if (TABLE) {
+        const int col = e0 + v;
+        if (col >= j0 && col < j0 + BW && col < p.cols)
+          static_cast<typename F::OutT*>(p.table)[row * p.table_pitch + col] = o;
+      }
+    }
+#pragma unroll
+    for (int v = 0; v < VP; ++v) {
+      cur[v] = nw_[v];
+      g[v] = gn[v];
+    }
+  }
+}
+
+template <class F, int VP, int HB, int D, bool TABLE>
+__global__ void __launch_bounds__(256) prevrow_cb_kernel(const FillParams p) {
+  using T = typename F::T;
+  using G = typename F::GridT;
+  static_assert(!(F::kMask & NB_L), "prev-row category: f must not read L");
+  static_assert(sizeof(T) == 4 && sizeof(G) == 4, "32-bit cells and costs");
+  static_assert(VP % 4 == 0 && HB % VP == 0, "16-byte lane segments; halos made of whole lanes");
+  constexpr int EXT = 32 * VP;
+  constexpr int BW = EXT - 2 * HB;
+  constexpr int HL = HB / VP;            // lanes per halo
+  static_assert(BW >= 2 * HB, "each edge publishes HB own columns");
+
+  extern __shared__ __align__(128) unsigned char cb_smem[];
+  const int lane = threadIdx.x & 31;
+  const int wl = threadIdx.x >> 5;
+  const int nw = blockDim.x >> 5;
+  const int q = blockIdx.x * nw + wl;   // column block
+  const int nb = p.nblocks;
+  Control* ctl = static_cast<Control*>(p.ctl);
+  const int W = p.cols;
+  const int64_t H = p.rows;
+
+  if (q < nb && H > 0) {
+    G* ring = reinterpret_cast<G*>(cb_smem) + (size_t)wl * D * EXT + lane * VP;   // this lane's columns
+    const int j0 = q * BW;
+    const int e0 = j0 - HB + lane * VP;   // first column of this lane
+    const G* cost = static_cast<const G*>(p.grid);
+    // out-of-table columns keep the boundary value of f in every row
+    uint32_t omask = 0;
+    T outv[VP];
+#pragma unroll
+    for (int v = 0; v < VP; ++v) {
+      const int col = e0 + v;
+      if (col < 0 || col >= W) omask |= 1u << v;
+      outv[v] = col < 0 ? F::left(p, 0) : F::right(p, 0);
+    }
+    const bool anyout = __any_sync(0xffffffffu, omask != 0);
+    // 16-byte segments of this lane: all in or all out (W % 4 == 0, e0 % 4 == 0)
+    uint32_t ssz[VP / 4];
+    const G* src[VP / 4];
+#pragma unroll
+    for (int s = 0; s < VP / 4; ++s) {
+      const int col = e0 + 4 * s;
+      const bool in = col >= 0 && col < W;
+      ssz[s] = in ? 16u : 0u;
+      asm volatile("mov.b32 %0, %0;" : "+r"(ssz[s]));   // opaque: no per-row rematerialisation
+      src[s] = cost + (in ? col : 0);
+    }
+    int ileft = (int)H;   // rows still to issue
+    uint32_t idst = smem_u32(ring);
+    int cslot = 0;
+#pragma unroll 1
+    for (int k = 0; k < D - 1; ++k) {
+      if (ileft > 0) {
+#pragma unroll
+        for (int s = 0; s < VP / 4; ++s) {
+          cb_cp16s(idst + 16 * s, src[s], ssz[s]);
+          src[s] += p.grid_pitch;
+        }
+      }
+      --ileft;
+      idst += EXT * 4;
+      cp_async_commit();
+    }
+
+    // costs of row 0 (the band loop loads row r+1 while computing row r)
+    G g[VP];
+    cp_async_wait_group<D - 2>();
+#pragma unroll
+    for (int s = 0; s < VP / 4; ++s) {
+      const int4 t = *reinterpret_cast<const int4*>(ring + 4 * s);
+      g[4 * s] = t.x; g[4 * s + 1] = t.y; g[4 * s + 2] = t.z; g[4 * s + 3] = t.w;
+    }
+
+    // row -1 (virtual): f's top initialisation
+    T cur[VP];
+#pragma unroll
+    for (int v = 0; v < VP; ++v) cur[v] = ((omask >> v) & 1u) ? outv[v] : F::top(p, e0 + v);
+
+    const uint32_t tag0 = (uint32_t)(p.epoch * 0x9E3779B1ull);
+    uint64_t* edges = reinterpret_cast<uint64_t*>(p.bnd);   // [nb][4 slots][2 sides][HB] pairs
+    const bool lhalo = lane < HL, rhalo = lane >= 32 - HL;
+    const bool ledge = lane >= HL && lane < 2 * HL;          // own columns [j0, j0 + HB)
+    const bool redge = lane >= 32 - 2 * HL && lane < 32 - HL; // own columns [j0 + BW - HB, j0 + BW)
+
+#pragma unroll 1
+    for (int64_t r0 = 0; r0 < H; r0 += HB) {
+      const int nr = (int)((H - r0 < HB) ? (H - r0) : HB);
+      if (anyout)
+        cb_band<F, VP, D, TABLE, true>(p, cur, g, nr, r0, ring, cslot, idst, ileft, src, ssz, outv, omask, e0, j0, BW);
+      else
+        cb_band<F, VP, D, TABLE, false>(p, cur, g, nr, r0, ring, cslot, idst, ileft, src, ssz, outv, omask, e0, j0, BW);
+      if (r0 + HB >= H) break;   // last band: outputs below
+      // ---- band boundary: publish own edges, take the neighbours' as halos
+      const int band = (int)(r0 / HB);
+      const uint32_t tag = tag0 + (uint32_t)band + 1u;
+      uint64_t* mine = edges + ((size_t)q * 4 + (band & 3)) * 2 * HB;
+      if (ledge || redge) {
+        uint64_t* d = mine + (ledge ? 0 : HB) + (ledge ? (lane - HL) : (lane - (32 - 2 * HL))) * VP;
+#pragma unroll
+        for (int v = 0; v < VP; v += 2)
+          cb_st_pair2(d + v, ((uint64_t)tag << 32) | (uint32_t)cur[v], ((uint64_t)tag << 32) | (uint32_t)cur[v + 1]);
+      }
+      const int nbq = lhalo ? q - 1 : q + 1;
+      const bool need = (lhalo && q > 0) || (rhalo && q + 1 < nb);
+      const uint64_t* s = nullptr;
+      if (need)
+        s = edges + ((size_t)nbq * 4 + (band & 3)) * 2 * HB + (lhalo ? HB + lane * VP : (lane - (32 - HL)) * VP);
+      uint64_t pr[VP];
+      bool ok = true;
+      if (need) {
+#pragma unroll
+        for (int v = 0; v < VP; v += 2) cb_ld_pair2(s + v, pr[v], pr[v + 1]);
+#pragma unroll
+        for (int v = 0; v < VP; ++v) ok = ok && ((uint32_t)(pr[v] >> 32) == tag);
+      }
+      if (!__all_sync(0xffffffffu, ok)) {
+        Backoff bo;
+        int spins = 0;
+        while (true) {
+          if (!ok) {
+            ok = true;
+#pragma unroll
+            for (int v = 0; v < VP; v += 2) cb_ld_pair2(s + v, pr[v], pr[v + 1]);
+#pragma unroll
+            for (int v = 0; v < VP; ++v) ok = ok && ((uint32_t)(pr[v] >> 32) == tag);
+          }
+          if (__all_sync(0xffffffffu, ok)) break;
+          // busy-poll first (the neighbour is normally within an L2 round trip), then back off
+          if (++spins > 64 && !bo.tick(ctl, p.timeout_ns)) return;
+        }
+      }
+      if (need) {
+#pragma unroll
+        for (int v = 0; v < VP; ++v) cur[v] = (T)(uint32_t)pr[v];
+      }
+    }
+    cp_async_wait_group<0>();
+
+    // ---- outputs of the last row
+    T mn = INT_MAX;
+#pragma unroll
+    for (int v = 0; v < VP; ++v) {
+      const int col = e0 + v;
+      if (col >= j0 && col < j0 + BW && col < W) {
+        if (p.last_row != nullptr) static_cast<T*>(p.last_row)[col] = cur[v];
+        mn = min(mn, cur[v]);
+      }
+    }
+    if (F::kScore == SCORE_ROW_MIN && p.score != nullptr) {
+      unsigned* rowmin_done = &ctl->pad[0];
+      T* rowmins = reinterpret_cast<T*>(p.prog);
+#pragma unroll
+      for (int off = 16; off > 0; off >>= 1) mn = min(mn, __shfl_xor_sync(0xffffffffu, mn, off));
+      if (lane == 0) {
+        rowmins[q] = mn;
+        __threadfence();
+        const unsigned d = atomicAdd(rowmin_done, 1u);
+        if (d == (unsigned)nb - 1) {
+          __threadfence();
+          T best = INT_MAX;
+          for (int k = 0; k < nb; ++k) best = min(best, __ldcg(rowmins + k));
+          *static_cast<T*>(p.score) = best;
+          atomicExch(rowmin_done, 0u);
+        }
+      }
+    }
+  }
+}
+
+// ---------------------------------------------------------------------------------------------
+// Compiled geometries: variant id -> (VP, HB, D); BW = 32*VP - 2*HB own columns per warp.
+template <class F, int VP, int HB, int D>
+static cudaError_t cb_launch(const FillParams& p, int nw, bool query, int* out, cudaStream_t s) {
+  const size_t smem = (size_t)nw * D * 32 * VP * sizeof(typename F::GridT);
+  auto kt = prevrow_cb_kernel<F, VP, HB, D, true>;
+  auto kf = prevrow_cb_kernel<F, VP, HB, D, false>;
+  cudaError_t e = cudaFuncSetAttribute(kt, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e == cudaSuccess) e = cudaFuncSetAttribute(kf, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  auto k = p.table != nullptr ? kt : kf;
+  if (query) {   // out = {own columns per warp, co-resident CTAs per SM}
+    int occ = 0;
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k, nw * 32, smem);
+    out[0] = 32 * VP - 2 * HB;
+    out[1] = occ;
+    return e;
+  }
+  const int grid = (p.nblocks + nw - 1) / nw;
+  FillParams pp = p;
+  void* args[] = {&pp};
+  return cudaLaunchCooperativeKernel((const void*)k, dim3(grid), dim3(nw * 32), args, smem, s);
+}
+
+template <class F>
+static cudaError_t cb_dispatch(int variant, const FillParams& p, int nw, bool query, int* out, cudaStream_t s) {
+  switch (variant) {
+    case 0: return cb_launch<F, 8, 64, 48>(p, nw, query, out, s);   // BW 128
+    case 1: return cb_launch<F, 8, 32, 48>(p, nw, query, out, s);
+    case 2: return cb_launch<F, 12, 48, 40>(p, nw, query, out, s);
+    case 3: return cb_launch<F, 16, 64, 32>(p, nw, query, out, s);
+    case 4: return cb_launch<F, 8, 64, 96>(p, nw, query, out, s);
+    case 5: return cb_launch<F, 4, 32, 64>(p, nw, query, out, s);   // BW 64
+    default: return cudaErrorInvalidValue;
+  }
+}
+
+// query = true: out[0] = own columns per warp (BW), out[1] = co-resident CTAs per SM.
+cudaError_t launch_prevrow_cb(int func, int variant, const FillParams& p, int nw, bool query, int* out,
+                              cudaStream_t s) {
+  switch (func) {
+    case 3: return cb_dispatch<CellMinPath3>(variant, p, nw, query, out, s);
+    case 4: return cb_dispatch<CellDiagMaxPlus>(variant, p, nw, query, out, s);
+    case 5: return cb_dispatch<CellMin2Plus>(variant, p, nw, query, out, s);
+    default: return cudaErrorInvalidValue;
+  }
+}
+
+}  // namespace lddp
