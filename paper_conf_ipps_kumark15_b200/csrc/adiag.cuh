@@ -34,10 +34,13 @@
 
 namespace lddp {
 
-#ifndef LDDP_AD_GUNROLL
-#define LDDP_AD_GUNROLL 1
+// 8-step groups per loop iteration (measured on B200: LCS / Levenshtein 2, DTW 4 -- C5 8.36 ->
+// 7.86 ms, C2 1.13 -> 1.00 ms against 1; LDDP_AD_GUNROLL overrides for experiments)
+#ifdef LDDP_AD_GUNROLL
+template <class F> constexpr int kAdGroupUnroll = LDDP_AD_GUNROLL;
+#else
+template <class F> constexpr int kAdGroupUnroll = F::kMatchCells ? 2 : 4;
 #endif
-constexpr int kAdGroupUnroll = LDDP_AD_GUNROLL;   // 8-step groups per loop iteration
 constexpr int kAdRing = 8;   // chunks (of 32 entries) per intra-CTA ring
 constexpr int kAdCRing = 256;  // per-warp column-context ring (entries), index = column & 255,
                                // plus an 8-entry overhang mirroring slots 0..7 (no wrap per step)
@@ -164,10 +167,13 @@ struct AdWarp {
     if (__all_sync(0xffffffffu, (uint32_t)(tp >> 32) == tag)) return true;
     const long long t0 = clock64();
     Backoff w;
+    int spins = 0;
     while (true) {
       if ((uint32_t)(tp >> 32) != tag) tp = (TS == 1) ? ad_ld_smem(src) : ad_ld_gpu(src);
       if (__all_sync(0xffffffffu, (uint32_t)(tp >> 32) == tag)) break;
-      if (!w.tick(ctl, p.timeout_ns)) return false;
+      // busy-poll first (a mid-strip wait is normally one hop of latency: sleeping there adds to
+      // the pipeline lag of every warp below), then back off
+      if (++spins > p.spin_polls && !w.tick(ctl, p.timeout_ns)) return false;
     }
     wait_top += clock64() - t0;
     return true;
@@ -225,7 +231,7 @@ struct AdWarp {
     }
     cpend = colctx_guard(p, 32 * (k + 2) + lane);
     __syncwarp();
-#pragma unroll kAdGroupUnroll
+#pragma unroll(kAdGroupUnroll<F>)
     for (int g = 0; g < 4; ++g) {
       CC cnext[8];
       const int tau0 = 32 * k - E + 8 * g;

@@ -145,7 +145,7 @@ LDDP_AD_TABLE_ROWS
 struct AdModel { double ipc, lat; };
 AdModel ad_model(int func) {
   switch (func) {
-    case LDDP_F_DTW: return {4.0, 9.0};          // FADD, FMNMX3, FADD; chain FMNMX3 -> FADD
+    case LDDP_F_DTW: return {6.0, 4.0};          // FADD, FMNMX3, FADD; refit with the 4-group unroll (C2: R4 E2 best)
     case LDDP_F_LEVENSHTEIN: return {4.6, 14.0}; // ISETP, VIMNMX3, IMAD, SEL; chain of three
     default: return {4.2, 4.5};                  // LCS: ISETP, IMAD, IMAD.MOV, VIMNMX3; chain VIMNMX3
   }
@@ -349,6 +349,7 @@ void fill_common(lddp_plan_t pl, const lddp_inputs* in, const lddp_outputs* out,
   p.halo = kPrevBandRows;
   p.nblocks = pl->nblocks;
   p.debug = env_int("LDDP_DEBUG", 0);
+  p.spin_polls = env_int("LDDP_SPIN", 256);
   p.one = 1;
   // debug trace buffer: LDDP_TRACE=<device pointer as decimal>:<chunks per row>
   if (const char* tr = getenv("LDDP_TRACE")) {
@@ -502,6 +503,8 @@ lddp_status lddp_plan(const lddp_desc* desc, lddp_plan_t* out) {
         if (Wq > 0 && g.W != Wq) continue;
         double c = ad_cost(d.func, g.R, g.E, g.W, d.rows, std::max<int64_t>(d.cols, 1), pl->sms);
         if (Rq > 0) c += 1e200 * std::abs(g.R - Rq);   // nearest compiled R to the request
+        if (getenv("LDDP_PLAN_DEBUG"))
+          fprintf(stderr, "[lddp plan] f=%d R=%d E=%d W=%d cost=%.0f\n", (int)d.func, g.R, g.E, g.W, c);
         if (c < best) { best = c; pl->R = g.R; pl->E = g.E; pl->W = g.W; pl->ad_launch = g.launch; }
       }
       if (pl->R == 0) {

@@ -51,6 +51,7 @@ struct FillParams {
   uint64_t* trace;
   int32_t trace_chunks;     // chunks per (strip, warp) row of the trace
   int32_t one;              // always 1 (a run-time constant the compiler cannot fold)
+  int32_t spin_polls;       // polls before a waiting warp starts to back off (env LDDP_SPIN)
   int32_t debug;            // env LDDP_DEBUG bits (development): 1 = adiag warps without handoffs
 };
 
