@@ -1,0 +1,256 @@
+// fsk.cu -- lane-systolic persistent kernel for Floyd-Steinberg dithering in the knight-move
+// category (t = 2i + j, Fig. 2 [L117-L122], Table I row "Y Y Y Y" [L140]; the FS algorithm of
+// §VI.B [L341] with the dependency constraint [L343-L344]).  The default FS kernel when the image
+// width and row pitch are multiples of 16 bytes (wavefront.cuh is the fallback).
+//
+//  * STRIPS of SH = 32*W rows (top-aligned; rows >= H are computed but never stored).  A CTA of W
+//    warps claims strips in increasing order; lane k of warp w owns ONE row i and processes
+//    column c = tau - D*k at warp step tau, D = 2 + E: the knight-move skew of 2 columns per row
+//    plus E steps of slack for the rotate SHFL that carries the error row to the lane below.
+//  * Lane k receives e(i-1, .) from lane k-1 through that one SHFL per step into a register FIFO:
+//    UR = fifo[E], U = fifo[E+1], UL = fifo[E+2]; L is the lane's own previous error.  Lane 31
+//    injects the warp's top row (the previous warp's bottom row) into the same SHFL.
+//  * Pixel arithmetic = CellFS::f, the oracle's pull form and operation order
+//    ((((in + e_UL/16) + e_U*5/16) + e_UR*3/16) + e_L*7/16, threshold 128, e = v - out), built
+//    with --fmad=false: bit-exact.  Absent neighbours are errors of +0 (v + (+0) == v exactly).
+//  * Image rows stream through a per-lane shared ring of 16-byte chunks (cp.async, 6 chunks
+//    ahead); output bytes are collected in a per-lane 4-chunk ring and stored 16 bytes at a time.
+//  * Warp and strip handoffs of the error rows are the adiag protocol (adiag.cuh): tagged
+//    (value, tag) pairs in a shared ring (warp w -> w+1) or in global memory (strip s -> s+1),
+//    validated per 32-column chunk; no flags, no fences.
+#include <cstdint>
+#include <climits>
+#include "adiag.cuh"
+
+namespace lddp {
+
+namespace {
+constexpr int kFsIn = 8;     // input chunks (16 B) per lane ring
+constexpr int kFsAhead = 6;  // chunks issued ahead of the lane's current chunk
+constexpr int kFsOut = 4;    // output chunks per lane ring
+
+__device__ __forceinline__ void fs_cp16(uint32_t dst, const void* src, uint32_t src_bytes) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src), "r"(src_bytes) : "memory");
+}
+}  // namespace
+
+template <int W, int E>
+__global__ void __launch_bounds__(W * 32, 1) fsk_kernel(const FillParams p) {
+  constexpr int D = 2 + E;
+  constexpr int SH = W * 32;
+  using F = CellFS;
+  __shared__ __align__(16) uint64_t ring[W][kAdRing][32];     // top stream of warp w >= 1
+  __shared__ int cons[W];
+  __shared__ __align__(16) float stg[W][32];                   // bottom staging row
+  __shared__ __align__(16) uint8_t inr[W][32][kFsIn][16];      // per-lane input chunks
+  __shared__ __align__(16) uint8_t outr[W][32][kFsOut][16];    // per-lane output chunks
+  __shared__ int strip_sh;
+
+  Control* ctl = static_cast<Control*>(p.ctl);
+  const int lane = threadIdx.x & 31;
+  const int wid = threadIdx.x >> 5;
+  const int Wimg = p.cols;
+  const int64_t H = p.rows;
+  const int NQ = (Wimg + 31) / 32;
+  const int K = NQ + D + 1;   // chunks per strip: the last lane reaches column 32(NQ+1)-1
+  const uint32_t ep32 = (uint32_t)p.epoch;
+  const uint8_t* img = static_cast<const uint8_t*>(p.grid);
+  uint8_t* out = static_cast<uint8_t*>(p.table);
+
+  for (int i = threadIdx.x; i < W * kAdRing * 32; i += blockDim.x) (&ring[0][0][0])[i] = 0ull;
+  if (threadIdx.x < W) cons[threadIdx.x] = 0;
+  __syncthreads();
+
+  uint32_t iter = 0;
+  while (true) {
+    if (threadIdx.x == 0) {
+      int s = (int)atomicAdd(&ctl->claim, 1u);
+      if (ld_volatile_u32(&ctl->abort)) s = INT_MAX;
+      strip_sh = s;
+    }
+    __syncthreads();
+    const int s = strip_sh;
+    if (s >= p.nstrips) break;
+    const int64_t row = (int64_t)s * SH + wid * 32 + lane;
+    const bool rvalid = row < H;
+    const uint8_t* rin = img + (rvalid ? row : 0) * p.grid_pitch;
+    uint8_t* rout = out + (rvalid ? row : 0) * p.table_pitch;
+    const uint32_t inbase = smem_u32(&inr[wid][lane][0][0]);
+    const uint32_t base = iter * (uint32_t)NQ + 1u;
+
+    // ---- input prologue: chunks q0 .. q0 + kFsAhead - 1 of this lane's first column
+    const int c_first = -D - D * lane;
+    int nq = c_first >> 4;   // floor(c / 16) (arithmetic shift)
+    for (int a = 0; a < kFsAhead; ++a, ++nq) {
+      const bool in = rvalid && nq >= 0 && 16 * nq < Wimg;
+      fs_cp16(inbase + (nq & (kFsIn - 1)) * 16, rin + (in ? 16 * nq : 0), in ? 16u : 0u);
+      cp_async_commit();
+    }
+    cp_async_wait_group<kFsAhead - 3>();
+    __syncwarp();
+
+    // ---- links (the adiag protocol)
+    const int topsrc = (wid > 0) ? 1 : (s > 0 ? 2 : 0);
+    const bool last_strip = (s == p.nstrips - 1);
+    const int botsnk = (wid < W - 1) ? 1 : (last_strip ? 0 : 2);
+    uint64_t* ring_top = &ring[wid][0][0];
+    uint64_t* ring_bot = &ring[(wid + 1) % W][0][0];
+    const uint64_t* gprev = static_cast<const uint64_t*>(p.bnd) + (int64_t)(s - 1) * p.bnd_stride;
+    uint64_t* gmine = static_cast<uint64_t*>(p.bnd) + (int64_t)s * p.bnd_stride;
+    uint64_t tp = 0, tq1 = (topsrc == 2) ? ad_ld_gpu(gprev + lane) : 0ull;
+
+    float fifo[E + 3];
+#pragma unroll
+    for (int d = 0; d < E + 3; ++d) fifo[d] = 0.0f;
+    float eL = 0.0f;
+    bool ok = true;
+
+    for (int k = 0; k < K && ok; ++k) {
+      // publish bottom chunk k-1-D (staged by lane 31 during chunk k-1)
+      const int j = k - 1 - D;
+      if (botsnk != 0 && j >= 0 && j < NQ) {
+        __syncwarp();
+        const float v = stg[wid][lane];
+        __syncwarp();
+        if (botsnk == 1) {
+          const uint32_t tag = base + (uint32_t)j;
+          if (j >= kAdRing) {
+            Backoff bo;
+            while ((int)((uint32_t)ad_ld_smem_i32(&cons[wid + 1]) - (tag - kAdRing)) < 0)
+              if (!bo.tick(ctl, p.timeout_ns)) { ok = false; break; }
+          }
+          uint64_t* d = ring_bot + (j & (kAdRing - 1)) * 32 + lane;
+          asm volatile("st.volatile.shared.u64 [%0], %1;" ::"r"(smem_u32(d)), "l"(ad_pair(ad_bits(v), tag)) : "memory");
+        } else {
+          uint64_t* d = gmine + 32 * (int64_t)j + lane;
+          asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(d), "l"(ad_pair(ad_bits(v), ep32)) : "memory");
+        }
+      }
+      if (!__all_sync(0xffffffffu, ok)) { ok = false; break; }
+      // acquire top chunk k (columns 32k + lane)
+      if (k < NQ) {
+        if (topsrc == 0) {
+          tp = 0ull;   // row -1: errors 0
+        } else {
+          const uint64_t* src;
+          uint32_t tag;
+          if (topsrc == 1) {
+            src = ring_top + (k % kAdRing) * 32 + lane;
+            tag = base + (uint32_t)k;
+            tp = ad_ld_smem(src);
+          } else {
+            src = gprev + 32 * (int64_t)k + lane;
+            tag = ep32;
+            tp = tq1;
+            tq1 = (k + 1 < NQ) ? ad_ld_gpu(src + 32) : 0ull;
+          }
+          if (!__all_sync(0xffffffffu, (uint32_t)(tp >> 32) == tag)) {
+            Backoff bo;
+            int spins = 0;
+            while (true) {
+              if ((uint32_t)(tp >> 32) != tag) tp = (topsrc == 1) ? ad_ld_smem(src) : ad_ld_gpu(src);
+              if (__all_sync(0xffffffffu, (uint32_t)(tp >> 32) == tag)) break;
+              if (++spins > p.spin_polls && !bo.tick(ctl, p.timeout_ns)) { ok = false; break; }
+            }
+            if (!__all_sync(0xffffffffu, ok)) { ok = false; break; }
+          }
+          if (topsrc == 1 && lane == 0) ad_st_smem_i32(&cons[wid], (int)(base + (uint32_t)k));
+        }
+      } else {
+        tp = 0ull;   // columns >= n: injected values never reach a stored pixel
+      }
+      const float topv = ad_val<float>(tp);
+
+      // ---- 32 steps: tau = 32k - D + su (fully unrolled: the period test below is static)
+#pragma unroll
+      for (int g = 0; g < 4; ++g) {
+        float bv[8];
+#pragma unroll
+        for (int u = 0; u < 8; ++u) {
+          const int tau = 32 * k - D + 8 * g + u;
+          const int c = tau - D * lane;
+          const float in = (float)inr[wid][lane][(c >> 4) & (kFsIn - 1)][c & 15];
+          const float UR = fifo[E], U = fifo[E + 1], UL = fifo[E + 2];
+          uint8_t o;
+          float e = F::f(eL, UL, U, UR, 0, 0, in, 0, 0, 0, o);
+          e = ((unsigned)c < (unsigned)Wimg) ? e : 0.0f;   // columns -1 and W are errors 0
+          outr[wid][lane][(c >> 4) & (kFsOut - 1)][c & 15] = o;
+          eL = e;
+          bv[u] = e;
+          const float inj = __shfl_sync(0xffffffffu, topv, 8 * g + u);
+          const float sv = (lane == 31) ? inj : e;
+          const float rv = __shfl_sync(0xffffffffu, sv, (lane + 31) & 31);
+#pragma unroll
+          for (int d = E + 2; d > 0; --d) fifo[d] = fifo[d - 1];
+          fifo[0] = rv;
+          if ((tau & 15) == 15) {
+            // period end: flush the completed output chunk, issue the next input chunk
+            const int qd = ((c + 1) >> 4) - 1;
+            if (rvalid && qd >= 0 && 16 * qd < Wimg) {
+              const uint4 w4 = *reinterpret_cast<const uint4*>(&outr[wid][lane][qd & (kFsOut - 1)][0]);
+              *reinterpret_cast<uint4*>(rout + 16 * qd) = w4;
+            }
+            const bool in2 = rvalid && nq >= 0 && 16 * nq < Wimg;
+            fs_cp16(inbase + (nq & (kFsIn - 1)) * 16, rin + (in2 ? 16 * nq : 0), in2 ? 16u : 0u);
+            cp_async_commit();
+            ++nq;
+            cp_async_wait_group<kFsAhead - 3>();
+            __syncwarp();
+          }
+        }
+        if (lane == 31) {
+          uint4* d = reinterpret_cast<uint4*>(&stg[wid][8 * g]);
+          d[0] = make_uint4(ad_bits(bv[0]), ad_bits(bv[1]), ad_bits(bv[2]), ad_bits(bv[3]));
+          d[1] = make_uint4(ad_bits(bv[4]), ad_bits(bv[5]), ad_bits(bv[6]), ad_bits(bv[7]));
+        }
+      }
+    }
+    // the last staged bottom chunk (K - 1 - D)
+    if (ok && botsnk != 0) {
+      const int j = K - 1 - D;
+      if (j >= 0 && j < NQ) {
+        __syncwarp();
+        const float v = stg[wid][lane];
+        __syncwarp();
+        if (botsnk == 1) {
+          const uint32_t tag = base + (uint32_t)j;
+          if (j >= kAdRing) {
+            Backoff bo;
+            while ((int)((uint32_t)ad_ld_smem_i32(&cons[wid + 1]) - (tag - kAdRing)) < 0)
+              if (!bo.tick(ctl, p.timeout_ns)) break;
+          }
+          uint64_t* d = ring_bot + (j & (kAdRing - 1)) * 32 + lane;
+          asm volatile("st.volatile.shared.u64 [%0], %1;" ::"r"(smem_u32(d)), "l"(ad_pair(ad_bits(v), tag)) : "memory");
+        } else {
+          uint64_t* d = gmine + 32 * (int64_t)j + lane;
+          asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(d), "l"(ad_pair(ad_bits(v), ep32)) : "memory");
+        }
+      }
+    }
+    cp_async_wait_group<0>();
+    __syncthreads();
+    ++iter;
+  }
+  if (threadIdx.x == 0) {
+    __threadfence();
+    const unsigned d = atomicAdd(&ctl->done, 1u);
+    if (d == gridDim.x - 1) {
+      atomicExch(&ctl->claim, 0u);
+      atomicExch(&ctl->done, 0u);
+    }
+  }
+}
+
+// W warps per CTA (strip = 32 W rows), E = extra lane lag.  grid <= strips.
+cudaError_t launch_fsk(const FillParams& p, int W, int E, int grid, cudaStream_t s) {
+#define LDDP_FSK(w, e)                                                   \
+  if (W == w && E == e) {                                                \
+    fsk_kernel<w, e><<<grid, w * 32, 0, s>>>(p);                         \
+    return cudaGetLastError();                                           \
+  }
+  LDDP_FSK(4, 1) LDDP_FSK(4, 2) LDDP_FSK(2, 1) LDDP_FSK(2, 2)
+#undef LDDP_FSK
+  return cudaErrorInvalidValue;
+}
+
+}  // namespace lddp

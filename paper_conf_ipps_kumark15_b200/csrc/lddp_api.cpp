@@ -209,6 +209,10 @@ struct lddp_plan_s {
   int cb_variant;    // column-block persistent kernel (prevrow_cb.cu): -1 = not usable
   int cb_nw;         // warps per CTA
   int cb_nblocks;    // column blocks (one warp each)
+  // Floyd-Steinberg lane-systolic kernel (fsk.cu): used when the widths / pitches allow
+  bool fsk;
+  int fsk_W, fsk_E, fsk_nstrips;
+  int64_t fsk_bnd_stride;
   // workspace layout (bytes)
   size_t off_prog, off_bnd, ws_bytes;
   // own workspace + host-fill staging
@@ -364,7 +368,14 @@ void fill_common(lddp_plan_t pl, const lddp_inputs* in, const lddp_outputs* out,
 
 lddp_status launch(lddp_plan_t pl, const FillParams& p, cudaStream_t s) {
   cudaError_t e = cudaSuccess;
-  if (pl->kind == 0) {
+  if (pl->kind == 0 && pl->fsk && p.grid_pitch % 16 == 0 && p.table_pitch % 16 == 0 &&
+      ((reinterpret_cast<uintptr_t>(p.grid) | reinterpret_cast<uintptr_t>(p.table)) & 15) == 0) {
+    FillParams q = p;
+    q.nstrips = pl->fsk_nstrips;
+    q.bnd_stride = pl->fsk_bnd_stride;
+    e = lddp::launch_fsk(q, pl->fsk_W, pl->fsk_E, std::min(pl->sms, pl->fsk_nstrips), s);
+    if (e == cudaErrorInvalidValue) return fail(LDDP_ERR_UNSUPPORTED, "fsk W=%d E=%d not compiled", pl->fsk_W, pl->fsk_E);
+  } else if (pl->kind == 0) {
     int grid = std::min(pl->grid, p.nstrips);
     int r = wf_dispatch(pl->desc.func, 0, pl->variant, p.table != nullptr, &p, grid, s);
     if (r < 0) return fail(LDDP_ERR_UNSUPPORTED, "wavefront variant %d not compiled for f=%d", pl->variant, pl->desc.func);
@@ -563,6 +574,18 @@ lddp_status lddp_plan(const lddp_desc* desc, lddp_plan_t* out) {
       pl->off_prog = 64;
       pl->off_bnd = align_up(pl->off_prog + (size_t)std::max(pl->nstrips, 1) * 8, 256);
       pl->ws_bytes = pl->off_bnd + (size_t)std::max(pl->nstrips, 1) * pl->bnd_stride * cell_bytes(d.func);
+      // FS: the lane-systolic knight kernel (fsk.cu) when the width is a multiple of 16 bytes
+      // (16-byte image chunks); row pitches / alignment are checked per fill
+      pl->fsk = false;
+      if (knight && d.func == LDDP_F_FS_DITHER && table && d.cols > 0 && d.rows > 0 && d.cols % 16 == 0 &&
+          env_int("LDDP_FSK", 1)) {
+        pl->fsk = true;
+        pl->fsk_W = env_int("LDDP_FSK_W", 4);
+        pl->fsk_E = env_int("LDDP_FSK_E", 1);
+        pl->fsk_nstrips = (int)((d.rows + 32 * pl->fsk_W - 1) / (32 * pl->fsk_W));
+        pl->fsk_bnd_stride = ((d.cols + 31) / 32) * 32;   // (value, tag) pairs per boundary row
+        pl->ws_bytes = std::max(pl->ws_bytes, pl->off_bnd + (size_t)pl->fsk_nstrips * pl->fsk_bnd_stride * 8);
+      }
     } else if (d.category == LDDP_CAT_PREV_ROW) {
       pl->kind = 1;
       pl->nblocks = (int)((d.cols + kPrevBW - 1) / kPrevBW);
@@ -636,6 +659,16 @@ lddp_status lddp_plan_describe(lddp_plan_t pl, char* buf, size_t len) {
   if (pl == nullptr || buf == nullptr || len == 0) return fail(LDDP_ERR_INVALID_ARG, "NULL argument");
   static const char* kinds[] = {"wavefront", "prevrow", "invl", "adiag"};
   const bool cb = pl->kind == 1 && pl->cb_variant >= 0;
+  if (pl->kind == 0 && pl->fsk) {
+    snprintf(buf, len,
+             "{\"kernel\": \"fsk\", \"variant\": -1, \"rows_per_lane\": 1, \"skew\": 2, \"extra_lag\": %d, "
+             "\"warps\": %d, \"grid\": %d, \"sms\": %d, \"occupancy\": 1, \"strip_rows\": %d, "
+             "\"strips\": %d, \"chunks\": %d, \"blocks\": 0, \"bands\": 0, \"workspace_bytes\": %zu, "
+             "\"fallback\": \"wavefront variant %d when pitches are not 16-byte multiples\"}",
+             pl->fsk_E, pl->fsk_W, std::min(pl->sms, pl->fsk_nstrips), pl->sms, 32 * pl->fsk_W, pl->fsk_nstrips,
+             (int)(pl->fsk_bnd_stride / 32), pl->ws_bytes, pl->variant);
+    return LDDP_OK;
+  }
   snprintf(buf, len,
            "{\"kernel\": \"%s\", \"variant\": %d, \"rows_per_lane\": %d, \"skew\": %d, \"extra_lag\": %d, "
            "\"warps\": %d, \"grid\": %d, \"sms\": %d, \"occupancy\": %d, \"strip_rows\": %lld, "

@@ -63,6 +63,8 @@ cudaError_t launch_prevrow(int func, const FillParams& p, int grid, cudaStream_t
 // per warp, out[1] = co-resident CTAs per SM (nothing launched).
 cudaError_t launch_prevrow_cb(int func, int variant, const FillParams& p, int nw, bool query, int* out,
                               cudaStream_t stream);
+// Floyd-Steinberg lane-systolic knight kernel (fsk.cu): W warps per CTA, E extra lane lag.
+cudaError_t launch_fsk(const FillParams& p, int W, int E, int grid, cudaStream_t stream);
 cudaError_t launch_invl(int func, const FillParams& p, int grid, cudaStream_t stream);
 
 // Per-kernel occupancy query (blocks per SM) for the chosen configuration.
