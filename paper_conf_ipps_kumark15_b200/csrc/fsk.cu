@@ -42,6 +42,7 @@ __global__ void __launch_bounds__(W * 32, 1) fsk_kernel(const FillParams p) {
   __shared__ __align__(16) uint64_t ring[W][kAdRing][32];     // top stream of warp w >= 1
   __shared__ int cons[W];
   __shared__ __align__(16) float stg[W][32];                   // bottom staging row
+  __shared__ __align__(16) float tstg[W][32];                  // top row of the current chunk
   __shared__ __align__(16) uint8_t inr[W][32][kFsIn][16];      // per-lane input chunks
   __shared__ __align__(16) uint8_t outr[W][32][kFsOut][16];    // per-lane output chunks
   __shared__ int strip_sh;
@@ -86,8 +87,16 @@ __global__ void __launch_bounds__(W * 32, 1) fsk_kernel(const FillParams p) {
       fs_cp16(inbase + (nq & (kFsIn - 1)) * 16, rin + (in ? 16 * nq : 0), in ? 16u : 0u);
       cp_async_commit();
     }
-    cp_async_wait_group<kFsAhead - 3>();
+    cp_async_wait_group<kFsAhead - 4>();
     __syncwarp();
+    // inputs of the first 8 steps (the step loop loads the NEXT group's inputs one group ahead:
+    // LDS.U8 + I2F on the pixel chain cost ~40 cycles per step)
+    float inq[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      const int c = -D + u - D * lane;
+      inq[u] = (float)inr[wid][lane][(c >> 4) & (kFsIn - 1)][c & 15];
+    }
 
     // ---- links (the adiag protocol)
     const int topsrc = (wid > 0) ? 1 : (s > 0 ? 2 : 0);
@@ -159,17 +168,40 @@ __global__ void __launch_bounds__(W * 32, 1) fsk_kernel(const FillParams p) {
       } else {
         tp = 0ull;   // columns >= n: injected values never reach a stored pixel
       }
-      const float topv = ad_val<float>(tp);
+      // chunk k's top row -> shared memory; lane 31 reads its 8 injections per group with two
+      // broadcast LDS.128 one group ahead (a per-step SHFL was scheduled late by ptxas)
+      __syncwarp();
+      tstg[wid][lane] = ad_val<float>(tp);
+      __syncwarp();
+      float injq[8];
+      {
+        const float4 a0 = reinterpret_cast<const float4*>(&tstg[wid][0])[0];
+        const float4 a1 = reinterpret_cast<const float4*>(&tstg[wid][0])[1];
+        injq[0] = a0.x; injq[1] = a0.y; injq[2] = a0.z; injq[3] = a0.w;
+        injq[4] = a1.x; injq[5] = a1.y; injq[6] = a1.z; injq[7] = a1.w;
+      }
 
       // ---- 32 steps: tau = 32k - D + su (fully unrolled: the period test below is static)
 #pragma unroll
       for (int g = 0; g < 4; ++g) {
         float bv[8];
+        float inn[8], injn[8];
+        if (g < 3) {
+          const float4 a0 = reinterpret_cast<const float4*>(&tstg[wid][8 * g + 8])[0];
+          const float4 a1 = reinterpret_cast<const float4*>(&tstg[wid][8 * g + 8])[1];
+          injn[0] = a0.x; injn[1] = a0.y; injn[2] = a0.z; injn[3] = a0.w;
+          injn[4] = a1.x; injn[5] = a1.y; injn[6] = a1.z; injn[7] = a1.w;
+        }
+#pragma unroll
+        for (int u = 0; u < 8; ++u) {
+          const int cn = 32 * k - D + 8 * g + 8 + u - D * lane;
+          inn[u] = (float)inr[wid][lane][(cn >> 4) & (kFsIn - 1)][cn & 15];
+        }
 #pragma unroll
         for (int u = 0; u < 8; ++u) {
           const int tau = 32 * k - D + 8 * g + u;
           const int c = tau - D * lane;
-          const float in = (float)inr[wid][lane][(c >> 4) & (kFsIn - 1)][c & 15];
+          const float in = inq[u];
           const float UR = fifo[E], U = fifo[E + 1], UL = fifo[E + 2];
           uint8_t o;
           float e = F::f(eL, UL, U, UR, 0, 0, in, 0, 0, 0, o);
@@ -177,7 +209,7 @@ __global__ void __launch_bounds__(W * 32, 1) fsk_kernel(const FillParams p) {
           outr[wid][lane][(c >> 4) & (kFsOut - 1)][c & 15] = o;
           eL = e;
           bv[u] = e;
-          const float inj = __shfl_sync(0xffffffffu, topv, 8 * g + u);
+          const float inj = injq[u];
           const float sv = (lane == 31) ? inj : e;
           const float rv = __shfl_sync(0xffffffffu, sv, (lane + 31) & 31);
 #pragma unroll
@@ -194,9 +226,14 @@ __global__ void __launch_bounds__(W * 32, 1) fsk_kernel(const FillParams p) {
             fs_cp16(inbase + (nq & (kFsIn - 1)) * 16, rin + (in2 ? 16 * nq : 0), in2 ? 16u : 0u);
             cp_async_commit();
             ++nq;
-            cp_async_wait_group<kFsAhead - 3>();
+            cp_async_wait_group<kFsAhead - 4>();
             __syncwarp();
           }
+        }
+#pragma unroll
+        for (int u = 0; u < 8; ++u) {
+          inq[u] = inn[u];
+          if (g < 3) injq[u] = injn[u];
         }
         if (lane == 31) {
           uint4* d = reinterpret_cast<uint4*>(&stg[wid][8 * g]);
@@ -248,7 +285,7 @@ cudaError_t launch_fsk(const FillParams& p, int W, int E, int grid, cudaStream_t
     fsk_kernel<w, e><<<grid, w * 32, 0, s>>>(p);                         \
     return cudaGetLastError();                                           \
   }
-  LDDP_FSK(4, 1) LDDP_FSK(4, 2) LDDP_FSK(2, 1) LDDP_FSK(2, 2)
+  LDDP_FSK(4, 0) LDDP_FSK(4, 1) LDDP_FSK(4, 2) LDDP_FSK(2, 0) LDDP_FSK(2, 1) LDDP_FSK(2, 2)
 #undef LDDP_FSK
   return cudaErrorInvalidValue;
 }

@@ -34,7 +34,7 @@ def fsk_env():
             os.environ[k] = v
 
 
-@pytest.mark.parametrize("w,e", [(4, 1), (4, 2), (2, 1), (2, 2)])
+@pytest.mark.parametrize("w,e", [(4, 0), (4, 1), (4, 2), (2, 0), (2, 1), (2, 2)])
 @pytest.mark.parametrize("shape", FS_SHAPES)
 @pytest.mark.parametrize("kind", ["ramp", "uniform"])
 def test_fsk_parity(fsk_env, w, e, shape, kind):
