@@ -136,6 +136,7 @@ struct AdWarp {
     const uint64_t* gprev;     // strip s-1's boundary row (TS 2)
     uint64_t* gmine;           // strip s's boundary row   (BS 2)
     T* stg;                    // this warp's bottom staging row (32 values, shared memory)
+    T* tstg;                   // this warp's top staging row: chunk k's 32 top values
     uint32_t base;             // ring chunk tag of chunk 0 in this strip
     uint32_t ep32;             // epoch tag of the global boundary pairs
     bool top_init;             // TS 0: the row above is table row 0 (else a virtual row)
@@ -218,7 +219,7 @@ struct AdWarp {
   // The 8-step body is identical for every warp role (no role branches inside it), so ptxas
   // can overlap consecutive steps and the body stays small for the instruction cache.
   template <bool CHECKED>
-  __device__ __forceinline__ void chunk(const FillParams& p, const int lane, const int k, T* stg) {
+  __device__ __forceinline__ void chunk(const FillParams& p, const int lane, const int k, T* stg, T* tstg) {
     const int n = p.cols;
     const int lane_off = lane * E;
     const T topv = ad_val<T>(tp);
@@ -230,7 +231,18 @@ struct AdWarp {
       if (slot < 8) cring[slot + kAdCRing] = cpend;
     }
     cpend = colctx_guard(p, 32 * (k + 2) + lane);
+    // chunk k's top row -> shared memory; lane 31 takes its 8 injections per group from there,
+    // loaded one group ahead (off the rotate-SHFL chain)
     __syncwarp();
+    tstg[lane] = topv;
+    __syncwarp();
+    T injq[8];
+    {
+      const uint4 i0 = reinterpret_cast<const uint4*>(tstg)[0];
+      const uint4 i1 = reinterpret_cast<const uint4*>(tstg)[1];
+      injq[0] = ad_val<T>(i0.x); injq[1] = ad_val<T>(i0.y); injq[2] = ad_val<T>(i0.z); injq[3] = ad_val<T>(i0.w);
+      injq[4] = ad_val<T>(i1.x); injq[5] = ad_val<T>(i1.y); injq[6] = ad_val<T>(i1.z); injq[7] = ad_val<T>(i1.w);
+    }
 #pragma unroll(kAdGroupUnroll<F>)
     for (int g = 0; g < 4; ++g) {
       CC cnext[8];
@@ -242,6 +254,13 @@ struct AdWarp {
           if constexpr (F::kMatchCells) cnext[u] = CC(mtab[(uint32_t)cr[u] * 32 + lane]);
           else cnext[u] = cr[u];
         }
+      }
+      T injn[8];
+      if (g < 3) {
+        const uint4 i0 = reinterpret_cast<const uint4*>(tstg + 8 * g + 8)[0];
+        const uint4 i1 = reinterpret_cast<const uint4*>(tstg + 8 * g + 8)[1];
+        injn[0] = ad_val<T>(i0.x); injn[1] = ad_val<T>(i0.y); injn[2] = ad_val<T>(i0.z); injn[3] = ad_val<T>(i0.w);
+        injn[4] = ad_val<T>(i1.x); injn[5] = ad_val<T>(i1.y); injn[6] = ad_val<T>(i1.z); injn[7] = ad_val<T>(i1.w);
       }
       T bv[8];
 #pragma unroll
@@ -265,7 +284,7 @@ struct AdWarp {
           nw[r] = v;
         }
         bv[u] = nw[R - 1];
-        const T inj = __shfl_sync(0xffffffffu, topv, 8 * g + u);
+        const T inj = injq[u];
         const T sv = (lane == 31) ? inj : nw[R - 1];
         const T rv = __shfl_sync(0xffffffffu, sv, (lane + 31) & 31);
 #pragma unroll
@@ -275,7 +294,10 @@ struct AdWarp {
         for (int r = 0; r < R; ++r) hist[r] = nw[r];
       }
 #pragma unroll
-      for (int u = 0; u < 8; ++u) ccur[u] = cnext[u];
+      for (int u = 0; u < 8; ++u) {
+        ccur[u] = cnext[u];
+        if (g < 3) injq[u] = injn[u];
+      }
       if (lane == 31) {
         uint4* d = reinterpret_cast<uint4*>(stg + 8 * g);
         d[0] = make_uint4(ad_bits(bv[0]), ad_bits(bv[1]), ad_bits(bv[2]), ad_bits(bv[3]));
@@ -292,7 +314,7 @@ struct AdWarp {
     if (!acquire_top(p, lane, k, NQ, TS, lk, ctl)) return false;
     // ring chunk k is in registers now: release its slot to warp w-1
     if (TS == 1 && k < NQ && lane == 0) ad_st_smem_i32(lk.cons_self, (int)(lk.base + (uint32_t)k));
-    chunk<CHECKED>(p, lane, k, lk.stg);
+    chunk<CHECKED>(p, lane, k, lk.stg, lk.tstg);
     return true;
   }
 
@@ -325,6 +347,7 @@ __global__ void __launch_bounds__(W * 32, 1) adiag_kernel(const FillParams p) {
   __shared__ int cons[W];                                   // last chunk tag consumed by warp w
   __shared__ typename F::ColCtx cring[W][kAdCRing + 8];    // per-warp column-context rings
   __shared__ __align__(16) T stg[W][32];                   // per-warp bottom staging row
+  __shared__ __align__(16) T tstg[W][32];                  // per-warp top staging row
   __shared__ int strip_sh;
   __shared__ int one_sh;
   extern __shared__ __align__(16) uint8_t ad_dyn_smem[];    // match tables (W x 256 x 32 u8)
@@ -429,6 +452,7 @@ __global__ void __launch_bounds__(W * 32, 1) adiag_kernel(const FillParams p) {
     lk.gprev = static_cast<const uint64_t*>(p.bnd) + (int64_t)(s - 1) * p.bnd_stride;
     lk.gmine = static_cast<uint64_t*>(p.bnd) + (int64_t)s * p.bnd_stride;
     lk.stg = stg[wid];
+    lk.tstg = tstg[wid];
     lk.base = base;
     lk.ep32 = ep32;
     lk.top_init = (strip_top - 1 == -1);
