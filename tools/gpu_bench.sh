@@ -12,7 +12,7 @@ timeout -s KILL 900 python bench.py > gpurun_out/bench.json 2> gpurun_out/bench.
 timeout -s KILL 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches_c5.csv \
    python bench.py --steps 3 --warmup 3 --no-others --no-cpu > gpurun_out/ncu_launch.log 2>&1; echo "launch rc=$?" >> gpurun_out/ncu_launch.log
 for W in C5 C2 C3 C4 C1; do
-  K=adiag; [ $W = C3 ] && K=wavefront; [ $W = C4 ] && K=prevrow
+  K=adiag; [ $W = C3 ] && K=fsk; [ $W = C4 ] && K=prevrow_cb
   timeout -s KILL 600 ncu --set full --clock-control none --import-source on -k regex:$K -s 2 -c 1 \
      -o gpurun_out/prof_$W python tools/quick_time.py $W --reps 3 > gpurun_out/ncu_$W.log 2>&1
   echo "ncu $W rc=$?" >> gpurun_out/ncu_$W.log
