@@ -51,24 +51,25 @@ template <class F, int VP, int D, bool TABLE, bool OUT>
 __device__ __forceinline__ void cb_band(const FillParams& p, typename F::T (&cur)[VP], typename F::GridT (&g)[VP],
                                         const int nr, const int64_t r0,
                                         const typename F::GridT* ring, int& cslot, uint32_t& idst, int& ileft,
-                                        const typename F::GridT* (&src)[VP / 4], const uint32_t (&ssz)[VP / 4],
+                                        int64_t& ioff, const int64_t pitch,
+                                        const typename F::GridT* const (&src)[VP / 4], const uint32_t (&ssz)[VP / 4],
                                         const typename F::T (&outv)[VP], const uint32_t omask, const int e0,
                                         const int j0, const int BW) {
   using T = typename F::T;
   using G = typename F::GridT;
   constexpr int EXT = 32 * VP;
-  const int64_t pitch = p.grid_pitch;
   const uint32_t ibeg = smem_u32(ring), iend = ibeg + (D - 1) * EXT * 4;
 #pragma unroll 2
   for (int r = 0; r < nr; ++r) {
-    // issue row + D - 1 into the slot consumed last (32-bit shared address, wraps at the ring end)
+    // issue row + D - 1 into the slot consumed last (32-bit shared address, wraps at the ring end).
+    // The global address is formed into a fresh register from the lane's row-0 pointer and a
+    // running element offset: updating the LDGSTS address register in place made the next row
+    // wait on the copy's register read (long-scoreboard stalls on the pointer increment).
     if (ileft > 0) {
 #pragma unroll
-      for (int s = 0; s < VP / 4; ++s) {
-        cb_cp16s(idst + 16 * s, src[s], ssz[s]);
-        src[s] += pitch;
-      }
+      for (int s = 0; s < VP / 4; ++s) cb_cp16s(idst + 16 * s, src[s] + ioff, ssz[s]);
     }
+    ioff += pitch;
     --ileft;
     idst = (idst == iend) ? ibeg : idst + EXT * 4;
     cp_async_commit();
@@ -159,15 +160,16 @@ __global__ void __launch_bounds__(256) prevrow_cb_kernel(const FillParams p) {
     int ileft = (int)H;   // rows still to issue
     uint32_t idst = smem_u32(ring);
     int cslot = 0;
+    int64_t pitch = p.grid_pitch;
+    asm volatile("mov.b64 %0, %0;" : "+l"(pitch));   // held in a register, not reloaded per row
+    int64_t ioff = 0;                                 // element offset of the next row to issue
 #pragma unroll 1
     for (int k = 0; k < D - 1; ++k) {
       if (ileft > 0) {
 #pragma unroll
-        for (int s = 0; s < VP / 4; ++s) {
-          cb_cp16s(idst + 16 * s, src[s], ssz[s]);
-          src[s] += p.grid_pitch;
-        }
+        for (int s = 0; s < VP / 4; ++s) cb_cp16s(idst + 16 * s, src[s] + ioff, ssz[s]);
       }
+      ioff += pitch;
       --ileft;
       idst += EXT * 4;
       cp_async_commit();
@@ -197,10 +199,11 @@ __global__ void __launch_bounds__(256) prevrow_cb_kernel(const FillParams p) {
     for (int64_t r0 = 0; r0 < H; r0 += HB) {
       const int nr = (int)((H - r0 < HB) ? (H - r0) : HB);
       if (anyout)
-        cb_band<F, VP, D, TABLE, true>(p, cur, g, nr, r0, ring, cslot, idst, ileft, src, ssz, outv, omask, e0, j0, BW);
+        cb_band<F, VP, D, TABLE, true>(p, cur, g, nr, r0, ring, cslot, idst, ileft, ioff, pitch, src, ssz, outv, omask, e0, j0, BW);
       else
-        cb_band<F, VP, D, TABLE, false>(p, cur, g, nr, r0, ring, cslot, idst, ileft, src, ssz, outv, omask, e0, j0, BW);
+        cb_band<F, VP, D, TABLE, false>(p, cur, g, nr, r0, ring, cslot, idst, ileft, ioff, pitch, src, ssz, outv, omask, e0, j0, BW);
       if (r0 + HB >= H) break;   // last band: outputs below
+      if (p.debug & 8) continue;   // development: no band exchange (wrong results; timing only)
       // ---- band boundary: publish own edges, take the neighbours' as halos
       const int band = (int)(r0 / HB);
       const uint32_t tag = tag0 + (uint32_t)band + 1u;
