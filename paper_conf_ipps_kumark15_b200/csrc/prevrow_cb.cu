@@ -37,6 +37,34 @@ __device__ __forceinline__ void cb_cp16(void* dst, const void* src, uint32_t src
 __device__ __forceinline__ void cb_cp16s(uint32_t dst, const void* src, uint32_t src_bytes) {
   asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src), "r"(src_bytes) : "memory");
 }
+__device__ __forceinline__ void cb_tma_row(uint32_t dst, const void* src, uint32_t bytes, uint32_t bar) {
+  asm volatile("mbarrier.arrive.expect_tx.release.cta.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
+               "l"(src), "r"(bytes), "r"(bar)
+               : "memory");
+}
+__device__ __forceinline__ bool cb_bar_ready(uint32_t bar, uint32_t parity) {
+  uint32_t ok;
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "mbarrier.try_wait.parity.acquire.cta.shared::cta.b64 p, [%1], %2;\n\t"
+      "selp.u32 %0, 1, 0, p;\n\t}"
+      : "=r"(ok)
+      : "r"(bar), "r"(parity)
+      : "memory");
+  return ok != 0;
+}
+// Bulk (TMA) row stream state of one warp: lane 0 issues one cp.async.bulk per row for the
+// in-table part of the warp's extended window; completion on one mbarrier per ring slot.
+struct CbBulk {
+  uint32_t dst0;      // shared address of slot 0's first in-table column
+  uint32_t bytes;     // in-table bytes of the window (multiple of 16)
+  uint32_t bar0;      // shared address of slot 0's mbarrier
+  const void* src0;   // global address of row 0's first in-table column
+  int irow, islot;    // next row to issue and its slot
+  uint32_t cpar;      // phase parity of the slot being consumed
+};
+
 __device__ __forceinline__ void cb_st_pair2(uint64_t* p, uint64_t a, uint64_t b) {
   asm volatile("st.relaxed.gpu.global.v2.u64 [%0], {%1, %2};" ::"l"(p), "l"(a), "l"(b) : "memory");
 }
@@ -47,8 +75,8 @@ __device__ __forceinline__ void cb_ld_pair2(const uint64_t* p, uint64_t& a, uint
 // One band of nr <= HB rows.  OUT: this lane holds out-of-table columns (their value is f's
 // boundary value in every row: one extra select per cell, taken only by the two edge blocks'
 // edge lanes -- warp-uniform for every other warp).
-template <class F, int VP, int D, bool TABLE, bool OUT>
-__device__ __forceinline__ void cb_band(const FillParams& p, typename F::T (&cur)[VP], typename F::GridT (&g)[VP],
+template <class F, int VP, int D, bool TABLE, bool OUT, bool BULK>
+__device__ __forceinline__ void cb_band(CbBulk& bk, const int lane, const FillParams& p, typename F::T (&cur)[VP], typename F::GridT (&g)[VP],
                                         const int nr, const int64_t r0,
                                         const typename F::GridT* ring, int& cslot, uint32_t& idst, int& ileft,
                                         int64_t& ioff, const int64_t pitch,
@@ -65,17 +93,31 @@ __device__ __forceinline__ void cb_band(const FillParams& p, typename F::T (&cur
     // The global address is formed into a fresh register from the lane's row-0 pointer and a
     // running element offset: updating the LDGSTS address register in place made the next row
     // wait on the copy's register read (long-scoreboard stalls on the pointer increment).
-    if (ileft > 0) {
+    if constexpr (BULK) {
+      if (lane == 0 && bk.irow < p.rows)
+        cb_tma_row(bk.dst0 + bk.islot * EXT * 4, static_cast<const char*>(bk.src0) + (int64_t)bk.irow * pitch * 4,
+                   bk.bytes, bk.bar0 + bk.islot * 8);
+      ++bk.irow;
+      bk.islot = (bk.islot + 1 == D) ? 0 : bk.islot + 1;
+    } else {
+      if (ileft > 0) {
 #pragma unroll
-      for (int s = 0; s < VP / 4; ++s) cb_cp16s(idst + 16 * s, src[s] + ioff, ssz[s]);
+        for (int s = 0; s < VP / 4; ++s) cb_cp16s(idst + 16 * s, src[s] + ioff, ssz[s]);
+      }
+      ioff += pitch;
+      --ileft;
+      idst = (idst == iend) ? ibeg : idst + EXT * 4;
+      cp_async_commit();
+      cp_async_wait_group<D - 2>();    // the NEXT row's group has landed: load it now, use it next row
     }
-    ioff += pitch;
-    --ileft;
-    idst = (idst == iend) ? ibeg : idst + EXT * 4;
-    cp_async_commit();
-    cp_async_wait_group<D - 2>();    // the NEXT row's group has landed: load it now, use it next row
     G gn[VP];
     cslot = (cslot + 1 == D) ? 0 : cslot + 1;
+    if constexpr (BULK) {
+      if (cslot == 0) bk.cpar ^= 1u;
+      if (r0 + r + 1 < p.rows)
+        while (!cb_bar_ready(bk.bar0 + cslot * 8, bk.cpar)) {
+        }
+    }
     const G* gs = ring + cslot * EXT;
 #pragma unroll
     for (int s = 0; s < VP / 4; ++s) {
@@ -109,7 +151,7 @@ __device__ __forceinline__ void cb_band(const FillParams& p, typename F::T (&cur
   }
 }
 
-template <class F, int VP, int HB, int D, bool TABLE>
+template <class F, int VP, int HB, int D, bool TABLE, bool BULK>
 __global__ void __launch_bounds__(256) prevrow_cb_kernel(const FillParams p) {
   using T = typename F::T;
   using G = typename F::GridT;
@@ -163,21 +205,47 @@ __global__ void __launch_bounds__(256) prevrow_cb_kernel(const FillParams p) {
     int64_t pitch = p.grid_pitch;
     asm volatile("mov.b64 %0, %0;" : "+l"(pitch));   // held in a register, not reloaded per row
     int64_t ioff = 0;                                 // element offset of the next row to issue
-#pragma unroll 1
-    for (int k = 0; k < D - 1; ++k) {
-      if (ileft > 0) {
-#pragma unroll
-        for (int s = 0; s < VP / 4; ++s) cb_cp16s(idst + 16 * s, src[s] + ioff, ssz[s]);
+    CbBulk bk{};
+    if constexpr (BULK) {
+      const uint32_t wbase = smem_u32(reinterpret_cast<G*>(cb_smem) + (size_t)wl * D * EXT);
+      const int cs = max(j0 - HB, 0), ce = min(j0 - HB + EXT, W);
+      bk.dst0 = wbase + (uint32_t)(cs - (j0 - HB)) * 4u;
+      bk.bytes = (uint32_t)(ce - cs) * 4u;
+      bk.bar0 = smem_u32(reinterpret_cast<uint64_t*>(cb_smem + (size_t)nw * D * EXT * sizeof(G)) + wl * D);
+      bk.src0 = cost + cs;
+      if (lane == 0) {
+        for (int k = 0; k < D; ++k)
+          asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bk.bar0 + 8 * k) : "memory");
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
       }
-      ioff += pitch;
-      --ileft;
-      idst += EXT * 4;
-      cp_async_commit();
+      __syncwarp();
+      for (int k = 0; k < D - 1; ++k) {
+        if (lane == 0 && k < H)
+          cb_tma_row(bk.dst0 + k * EXT * 4, static_cast<const char*>(bk.src0) + (int64_t)k * pitch * 4, bk.bytes,
+                     bk.bar0 + k * 8);
+      }
+      bk.irow = D - 1;
+      bk.islot = D - 1;
+      bk.cpar = 0;
+      while (!cb_bar_ready(bk.bar0, 0u)) {
+      }
+    } else {
+#pragma unroll 1
+      for (int k = 0; k < D - 1; ++k) {
+        if (ileft > 0) {
+#pragma unroll
+          for (int s = 0; s < VP / 4; ++s) cb_cp16s(idst + 16 * s, src[s] + ioff, ssz[s]);
+        }
+        ioff += pitch;
+        --ileft;
+        idst += EXT * 4;
+        cp_async_commit();
+      }
+      cp_async_wait_group<D - 2>();
     }
 
     // costs of row 0 (the band loop loads row r+1 while computing row r)
     G g[VP];
-    cp_async_wait_group<D - 2>();
 #pragma unroll
     for (int s = 0; s < VP / 4; ++s) {
       const int4 t = *reinterpret_cast<const int4*>(ring + 4 * s);
@@ -199,9 +267,9 @@ __global__ void __launch_bounds__(256) prevrow_cb_kernel(const FillParams p) {
     for (int64_t r0 = 0; r0 < H; r0 += HB) {
       const int nr = (int)((H - r0 < HB) ? (H - r0) : HB);
       if (anyout)
-        cb_band<F, VP, D, TABLE, true>(p, cur, g, nr, r0, ring, cslot, idst, ileft, ioff, pitch, src, ssz, outv, omask, e0, j0, BW);
+        cb_band<F, VP, D, TABLE, true, BULK>(bk, lane, p, cur, g, nr, r0, ring, cslot, idst, ileft, ioff, pitch, src, ssz, outv, omask, e0, j0, BW);
       else
-        cb_band<F, VP, D, TABLE, false>(p, cur, g, nr, r0, ring, cslot, idst, ileft, ioff, pitch, src, ssz, outv, omask, e0, j0, BW);
+        cb_band<F, VP, D, TABLE, false, BULK>(bk, lane, p, cur, g, nr, r0, ring, cslot, idst, ileft, ioff, pitch, src, ssz, outv, omask, e0, j0, BW);
       if (r0 + HB >= H) break;   // last band: outputs below
       if (p.debug & 8) continue;   // development: no band exchange (wrong results; timing only)
       // ---- band boundary: publish own edges, take the neighbours' as halos
@@ -248,7 +316,7 @@ __global__ void __launch_bounds__(256) prevrow_cb_kernel(const FillParams p) {
         for (int v = 0; v < VP; ++v) cur[v] = (T)(uint32_t)pr[v];
       }
     }
-    cp_async_wait_group<0>();
+    if constexpr (!BULK) cp_async_wait_group<0>();
 
     // ---- outputs of the last row
     T mn = INT_MAX;
@@ -283,11 +351,11 @@ __global__ void __launch_bounds__(256) prevrow_cb_kernel(const FillParams p) {
 
 // ---------------------------------------------------------------------------------------------
 // Compiled geometries: variant id -> (VP, HB, D); BW = 32*VP - 2*HB own columns per warp.
-template <class F, int VP, int HB, int D>
+template <class F, int VP, int HB, int D, bool BULK = false>
 static cudaError_t cb_launch(const FillParams& p, int nw, bool query, int* out, cudaStream_t s) {
-  const size_t smem = (size_t)nw * D * 32 * VP * sizeof(typename F::GridT);
-  auto kt = prevrow_cb_kernel<F, VP, HB, D, true>;
-  auto kf = prevrow_cb_kernel<F, VP, HB, D, false>;
+  const size_t smem = (size_t)nw * D * 32 * VP * sizeof(typename F::GridT) + (BULK ? (size_t)nw * D * 8 : 0);
+  auto kt = prevrow_cb_kernel<F, VP, HB, D, true, BULK>;
+  auto kf = prevrow_cb_kernel<F, VP, HB, D, false, BULK>;
   cudaError_t e = cudaFuncSetAttribute(kt, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e == cudaSuccess) e = cudaFuncSetAttribute(kf, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
@@ -314,6 +382,8 @@ static cudaError_t cb_dispatch(int variant, const FillParams& p, int nw, bool qu
     case 3: return cb_launch<F, 16, 64, 32>(p, nw, query, out, s);
     case 4: return cb_launch<F, 8, 64, 96>(p, nw, query, out, s);
     case 5: return cb_launch<F, 4, 32, 64>(p, nw, query, out, s);   // BW 64
+    case 6: return cb_launch<F, 4, 32, 64, true>(p, nw, query, out, s);   // BW 64, TMA rows
+    case 7: return cb_launch<F, 8, 64, 48, true>(p, nw, query, out, s);   // BW 128, TMA rows
     default: return cudaErrorInvalidValue;
   }
 }

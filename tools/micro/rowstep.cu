@@ -11,17 +11,28 @@
 #include <cuda_runtime.h>
 
 template <int VP, int MODE>
-__global__ void __launch_bounds__(128, 1) rows(int n, int* out, long long* cyc) {
+__global__ void __launch_bounds__(128, 1) rows(int n, int* out, long long* cyc, const int* __restrict__ gsrc) {
   __shared__ __align__(16) int ring[4][8][32 * VP];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   for (int i = threadIdx.x; i < 4 * 8 * 32 * VP; i += blockDim.x) (&ring[0][0][0])[i] = i & 1023;
   __syncthreads();
   int cur[VP], gk[VP], gn[VP];
   for (int v = 0; v < VP; ++v) { cur[v] = lane + v; gk[v] = v; gn[v] = v; }
+  // MODE 5 / 6: + one 16-byte cp.async per lane per row from global (6: every 4th row commits)
+  __shared__ __align__(16) int cring[4][16][32 * 4];
+  const uint32_t cbase = (uint32_t)__cvta_generic_to_shared(&cring[w][0][lane * 4]);
   long long t0 = clock64();
   for (int r = 0; r < n; ++r) {
+    if (MODE >= 5) {
+      const int* src = gsrc + ((size_t)(r & 4095) * 32768 + blockIdx.x * 128 + threadIdx.x * 4);
+      asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(cbase + (r & 15) * 512), "l"(src) : "memory");
+      if (MODE == 5 || (r & 3) == 3) {
+        asm volatile("cp.async.commit_group;" ::: "memory");
+        asm volatile("cp.async.wait_group 14;" ::: "memory");
+      }
+    }
     int g[VP];
-    if (MODE == 1) {
+    if (MODE == 1 || MODE >= 5) {
 #pragma unroll
       for (int v = 0; v < VP; ++v) g[v] = gk[v] + (r & 1);
     } else if (MODE == 4) {
@@ -59,11 +70,10 @@ __global__ void __launch_bounds__(128, 1) rows(int n, int* out, long long* cyc) 
 }
 
 template <int VP, int MODE>
-void run(int* out, long long* cyc, int n) {
-  cudaFuncSetAttribute(rows<VP, MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, 0);
-  rows<VP, MODE><<<148, 128>>>(n, out, cyc);
+void run(int* out, long long* cyc, int n, const int* g) {
+  rows<VP, MODE><<<148, 128>>>(n, out, cyc, g);
   cudaDeviceSynchronize();
-  rows<VP, MODE><<<148, 128>>>(n, out, cyc);
+  rows<VP, MODE><<<148, 128>>>(n, out, cyc, g);
   cudaError_t e = cudaDeviceSynchronize();
   long long h[148 * 4];
   cudaMemcpy(h, cyc, sizeof(h), cudaMemcpyDeviceToHost);
@@ -79,12 +89,12 @@ int main() {
   cudaMalloc(&out, 148 * 128 * 4);
   cudaMalloc(&cyc, 148 * 4 * 8);
   const int n = 1 << 14;
-  run<4, 0>(out, cyc, n);
-  run<4, 1>(out, cyc, n);
-  run<4, 2>(out, cyc, n);
-  run<4, 3>(out, cyc, n);
-  run<4, 4>(out, cyc, n);
-  run<8, 0>(out, cyc, n);
-  run<8, 4>(out, cyc, n);
+  int* g;
+  cudaMalloc(&g, (size_t)4096 * 32768 * 4);
+  run<4, 0>(out, cyc, n, g);
+  run<4, 1>(out, cyc, n, g);
+  run<4, 4>(out, cyc, n, g);
+  run<4, 5>(out, cyc, n, g);
+  run<4, 6>(out, cyc, n, g);
   return 0;
 }
