@@ -87,8 +87,14 @@ __device__ __forceinline__ uint64_t ad_pair(uint32_t bits, uint32_t tag) {
   return ((uint64_t)tag << 32) | bits;
 }
 
-template <class F, int R, int W, int E>
+// S = 1 ("split"): the lane's rows [R/2, R) run one column behind rows [0, R/2) -- their U at
+// column c-1 is the upper half's value from the previous step -- so a step holds two independent
+// chains of R/2 cells (ILP 2) for one extra step of lane lag (ELAG = E + S).
+template <class F, int R, int W, int E, int S = 0>
 struct AdWarp {
+  static constexpr int ELAG = E + S;   // lane-to-lane column lag
+  static constexpr int H2 = S ? R / 2 : R;
+  static_assert(!S || (R % 2 == 0), "split needs an even R");
   using T = typename F::T;
   using RC = typename F::RowCtx;
   using CC = typename F::ColCtx;
@@ -103,6 +109,8 @@ struct AdWarp {
   T leftv[R];       // column -1 of each row
   T rlast[R];       // column n-1 of each row (captured in checked chunks)
   CC ccur[8];       // column contexts of the current 8-step group
+  CC cprv;          // split: context of the lower half's column (the previous step's)
+  T midUL;          // split: upper half's last row two steps back (UL of the lower half)
   CC cpend;         // column context of column 32(k+2) + lane, staged into the ring at chunk k+1
   CC* cring;        // this warp's column-context ring (shared memory)
   uint8_t* mtab;    // match cells: this warp's table mtab[c * 32 + lane] = rows r of the lane with
@@ -221,7 +229,7 @@ struct AdWarp {
   template <bool CHECKED>
   __device__ __forceinline__ void chunk(const FillParams& p, const int lane, const int k, T* stg, T* tstg) {
     const int n = p.cols;
-    const int lane_off = lane * E;
+    const int lane_off = lane * ELAG;
     const T topv = ad_val<T>(tp);
     // column contexts: one coalesced load per 32 columns, two chunks ahead, staged through the
     // warp's shared ring (the body reads it with LDS: lower latency than L1 hits)
@@ -270,18 +278,51 @@ struct AdWarp {
         T U = fifo[E - 1];
         T UL = fifo[E];
         T nw[R];
+        if constexpr (S) {
+          // upper half at column c, lower half at column c-1: two independent chains, interleaved
+          const int cl = c - 1;
+          T UB = hist[H2 - 1];   // upper row H2-1 at column c-1 (previous step)
+          T ULB = midUL;         // ... at column c-2
 #pragma unroll
-        for (int r = 0; r < R; ++r) {
-          T v;
-          if constexpr (F::kMatchCells) v = F::fadm(hist[r], UL, U, ((uint32_t)cc >> r) & 1u, one);
-          else v = F::fad(hist[r], UL, U, rc[r], cc, one);
-          if (CHECKED) {
-            v = (c == -1) ? leftv[r] : v;
-            rlast[r] = (c == n - 1) ? v : rlast[r];
+          for (int r = 0; r < H2; ++r) {
+            T v, w;
+            const int q = H2 + r;
+            if constexpr (F::kMatchCells) {
+              v = F::fadm(hist[r], UL, U, ((uint32_t)cc >> r) & 1u, one);
+              w = F::fadm(hist[q], ULB, UB, ((uint32_t)cprv >> q) & 1u, one);
+            } else {
+              v = F::fad(hist[r], UL, U, rc[r], cc, one);
+              w = F::fad(hist[q], ULB, UB, rc[q], cprv, one);
+            }
+            if (CHECKED) {
+              v = (c == -1) ? leftv[r] : v;
+              rlast[r] = (c == n - 1) ? v : rlast[r];
+              w = (cl == -1) ? leftv[q] : w;
+              rlast[q] = (cl == n - 1) ? w : rlast[q];
+            }
+            UL = hist[r];
+            U = v;
+            nw[r] = v;
+            ULB = hist[q];
+            UB = w;
+            nw[q] = w;
           }
-          UL = hist[r];
-          U = v;
-          nw[r] = v;
+          midUL = hist[H2 - 1];
+          cprv = cc;
+        } else {
+#pragma unroll
+          for (int r = 0; r < R; ++r) {
+            T v;
+            if constexpr (F::kMatchCells) v = F::fadm(hist[r], UL, U, ((uint32_t)cc >> r) & 1u, one);
+            else v = F::fad(hist[r], UL, U, rc[r], cc, one);
+            if (CHECKED) {
+              v = (c == -1) ? leftv[r] : v;
+              rlast[r] = (c == n - 1) ? v : rlast[r];
+            }
+            UL = hist[r];
+            U = v;
+            nw[r] = v;
+          }
         }
         bv[u] = nw[R - 1];
         const T inj = injq[u];
@@ -310,7 +351,7 @@ struct AdWarp {
   __device__ __forceinline__ bool step_chunk(const FillParams& p, const int lane, const int k, const int NQ,
                                              const int TS, const int BS, Links& lk, Control* ctl) {
     // the staging row holds bottom chunk k-1-E (produced during chunk k-1): publish it first
-    if (!publish_bottom(p, lane, k - 1 - E, NQ, BS, lk, ctl)) return false;
+    if (!publish_bottom(p, lane, k - 1 - ELAG, NQ, BS, lk, ctl)) return false;
     if (!acquire_top(p, lane, k, NQ, TS, lk, ctl)) return false;
     // ring chunk k is in registers now: release its slot to warp w-1
     if (TS == 1 && k < NQ && lane == 0) ad_st_smem_i32(lk.cons_self, (int)(lk.base + (uint32_t)k));
@@ -323,8 +364,8 @@ struct AdWarp {
   __device__ __forceinline__ bool strip(const FillParams& p, const int lane, const int NQ, const int TS,
                                         const int BS, Links& lk, Control* ctl) {
     const int n = p.cols;
-    const int K = NQ + E;
-    const int k0 = min(E, K);
+    const int K = NQ + ELAG;
+    const int k0 = min(ELAG, K);
     // steady: every lane's columns in [0, n-1) (no boundary column in the chunk)
     int k1 = (n - 33 + E) >= 0 ? (n - 33 + E) / 32 + 1 : 0;
     k1 = max(k0, min(K, k1));
@@ -334,13 +375,13 @@ struct AdWarp {
       if (!step_chunk<false>(p, lane, k, NQ, TS, BS, lk, ctl)) return false;
     for (int k = k1; k < K; ++k)
       if (!step_chunk<true>(p, lane, k, NQ, TS, BS, lk, ctl)) return false;
-    return publish_bottom(p, lane, K - 1 - E, NQ, BS, lk, ctl);   // the last staged chunk
+    return publish_bottom(p, lane, K - 1 - ELAG, NQ, BS, lk, ctl);   // the last staged chunk
   }
 };
 
-template <class F, int R, int W, int E>
+template <class F, int R, int W, int E, int S = 0>
 __global__ void __launch_bounds__(W * 32, 1) adiag_kernel(const FillParams p) {
-  using AW = AdWarp<F, R, W, E>;
+  using AW = AdWarp<F, R, W, E, S>;
   using T = typename AW::T;
   constexpr int SH = AW::SH;
   __shared__ __align__(16) uint64_t ring[W][kAdRing][32];   // ring[w]: top stream of warp w >= 1
@@ -395,13 +436,15 @@ __global__ void __launch_bounds__(W * 32, 1) adiag_kernel(const FillParams p) {
       aw.rlast[r] = T(0);
       aw.hist[r] = T(0);
     }
+    aw.midUL = T(0);
+    aw.cprv = typename F::ColCtx(0);
 #pragma unroll
     for (int d = 0; d <= E; ++d) aw.fifo[d] = T(0);
     // lane 0's UL at column 0: the row above the warp at column -1 (received "before" step -E)
     if (lane == 0) aw.fifo[0] = aw.leftval(p, wtop - 1);
     aw.cring = cring[wid];
     aw.one = ad_ld_smem_i32(&one_sh);   // a volatile load: ptxas cannot rematerialise it per use
-    for (int q = -E - 1; q <= 0; ++q) {
+    for (int q = -E - 1 - S; q <= 0; ++q) {
       const int slot = (32 * q + lane) & (kAdCRing - 1);
       const typename F::ColCtx v = aw.colctx_guard(p, 32 * q + lane);
       aw.cring[slot] = v;
@@ -423,7 +466,7 @@ __global__ void __launch_bounds__(W * 32, 1) adiag_kernel(const FillParams p) {
     }
 #pragma unroll
     for (int u = 0; u < 8; ++u) {
-      const typename F::ColCtx c = aw.cring[((-E - lane * E) & (kAdCRing - 1)) + u];
+      const typename F::ColCtx c = aw.cring[((-E - lane * AW::ELAG) & (kAdCRing - 1)) + u];
       if constexpr (F::kMatchCells) aw.ccur[u] = typename F::ColCtx(aw.mtab[(uint32_t)c * 32 + lane]);
       else aw.ccur[u] = c;
     }

@@ -129,7 +129,7 @@ int wf_dispatch(int func, int op, int variant, bool table, const FillParams* p, 
 
 // Compiled adiag geometries (tools/gen_adiag.py): f, rows per lane R, lane lag E, warps per CTA W.
 struct AdGeom {
-  int func, R, E, W;
+  int func, R, E, W, S;
   cudaError_t (*launch)(const FillParams&, int, cudaStream_t);
 };
 const AdGeom kAdGeoms[] = {
@@ -150,14 +150,16 @@ AdModel ad_model(int func) {
     default: return {4.2, 4.5};                  // LCS: ISETP, IMAD, IMAD.MOV, VIMNMX3; chain VIMNMX3
   }
 }
-double ad_cost(int func, int R, int E, int W, int64_t m, int64_t n, int sms) {
+double ad_cost(int func, int R, int E, int W, int S, int64_t m, int64_t n, int sms) {
   const AdModel md = ad_model(func);
   const double share = W / 4.0;   // warps per SM sub-partition
-  const double t = std::max((md.lat * R + 31.0) / E, share * md.ipc * R) + 12.0;
+  // split (S = 1): two independent chains of R/2 cells per step, one more step of lane lag
+  const double chain = md.lat * (S ? R / 2 : R) + 31.0;
+  const double t = std::max(chain / E, share * md.ipc * R * (S ? 0.8 : 1.0)) + 12.0;
   const int64_t warps = (m + 32 * R - 1) / (32 * R);
   const int64_t cap = (int64_t)W * sms;
   const int64_t waves = (warps + cap - 1) / cap;
-  const double lag = (double)warps * (32.0 * E + 12.0) + (double)((warps + W - 1) / W) * 40.0;
+  const double lag = (double)warps * (32.0 * (E + S) + 12.0) + (double)((warps + W - 1) / W) * 40.0;
   return ((double)waves * (double)n + lag) * t;
 }
 
@@ -506,23 +508,26 @@ lddp_status lddp_plan(const lddp_desc* desc, lddp_plan_t* out) {
       int Rq = d.tile_rows > 0 ? d.tile_rows : env_int("LDDP_AD_R", 0);
       int Eq = env_int("LDDP_AD_E", 0);
       int Wq = d.tile_warps > 0 ? d.tile_warps : env_int("LDDP_AD_W", 0);
+      int Sq = env_int("LDDP_AD_S", -1);
       double best = 1e300;
       pl->R = 0;
       for (const auto& g : kAdGeoms) {
         if (g.func != d.func) continue;
         if (Eq > 0 && g.E != Eq) continue;
         if (Wq > 0 && g.W != Wq) continue;
-        double c = ad_cost(d.func, g.R, g.E, g.W, d.rows, std::max<int64_t>(d.cols, 1), pl->sms);
+        if (Sq >= 0 && g.S != Sq) continue;
+        if (Sq < 0 && g.S) continue;   // split geometries only on request: measured slower on B200 (C5 6.9 -> 11.6 ms)
+        double c = ad_cost(d.func, g.R, g.E, g.W, g.S, d.rows, std::max<int64_t>(d.cols, 1), pl->sms);
         if (Rq > 0) c += 1e200 * std::abs(g.R - Rq);   // nearest compiled R to the request
         if (getenv("LDDP_PLAN_DEBUG"))
-          fprintf(stderr, "[lddp plan] f=%d R=%d E=%d W=%d cost=%.0f\n", (int)d.func, g.R, g.E, g.W, c);
-        if (c < best) { best = c; pl->R = g.R; pl->E = g.E; pl->W = g.W; pl->ad_launch = g.launch; }
+          fprintf(stderr, "[lddp plan] f=%d R=%d E=%d W=%d S=%d cost=%.0f\n", (int)d.func, g.R, g.E, g.W, g.S, c);
+        if (c < best) { best = c; pl->R = g.R; pl->E = g.E; pl->W = g.W; pl->SIG = g.S; pl->ad_launch = g.launch; }
       }
       if (pl->R == 0) {
         delete pl;
         return fail(LDDP_ERR_UNSUPPORTED, "no compiled adiag geometry for f=%d (E=%d W=%d)", d.func, Eq, Wq);
       }
-      pl->SIG = 0;
+      // pl->SIG carries the split flag (reported as "skew")
       pl->variant = -1;
       pl->occupancy = 1;
       pl->strip_rows = (int64_t)pl->W * 32 * pl->R;

@@ -42,10 +42,11 @@ def _check(func, got, ref):
             np.testing.assert_array_equal(g, r, err_msg=k)
 
 
-def _run(func, R, E, W, a, b, **kw):
-    old = {k: os.environ.get(k) for k in ("LDDP_AD_E", "LDDP_AD_W")}
+def _run(func, R, E, W, a, b, S=0, **kw):
+    old = {k: os.environ.get(k) for k in ("LDDP_AD_E", "LDDP_AD_W", "LDDP_AD_S")}
     os.environ["LDDP_AD_E"] = str(E)
     os.environ["LDDP_AD_W"] = str(W)
+    os.environ["LDDP_AD_S"] = str(S)
     try:
         got = run_gpu(func, "anti_diagonal", a=a, b=b, outputs=("score", "last_row", "last_col"),
                       tile_rows=R, **kw)
@@ -57,30 +58,32 @@ def _run(func, R, E, W, a, b, **kw):
                 os.environ[k] = v
     plan = got["plan"]
     assert '"adiag"' in plan and f'"rows_per_lane": {R},' in plan and f'"extra_lag": {E},' in plan, plan
-    assert f'"warps": {W},' in plan, plan
+    assert f'"warps": {W},' in plan and f'"skew": {S},' in plan, plan
     return got
 
 
 def _cases():
     for func, geoms in GEOMS.items():
-        for R, E, W in geoms:
+        for geom in geoms:
+            R, E, W = geom[:3]
+            S = geom[3] if len(geom) > 3 else 0   # split: lower half of the rows one column behind
             sh = 32 * W * R
             for m, n in [(1, 1), (1, 70), (70, 1), (sh - 1, 33), (sh, 32), (sh + 1, 31), (2 * sh + 5, 41),
                          (3 * sh - 7, 72), (sh // 2 + 3, 1000), (997, 1009)]:
-                yield func, R, E, W, m, n
+                yield func, R, E, W, S, m, n
 
 
-@pytest.mark.parametrize("func,R,E,W,m,n", list(_cases()))
-def test_adiag_geometry(func, R, E, W, m, n):
+@pytest.mark.parametrize("func,R,E,W,S,m,n", list(_cases()))
+def test_adiag_geometry(func, R, E, W, S, m, n):
     a, b = _inputs(func, 31 * m + n + R, m, n)
-    _check(func, _run(func, R, E, W, a, b), _ref(func, a, b))
+    _check(func, _run(func, R, E, W, a, b, S=S), _ref(func, a, b))
 
 
 @pytest.mark.parametrize("func", ["lcs", "levenshtein", "dtw"])
 @pytest.mark.parametrize("grid", [1, 2, 3])
 def test_adiag_small_grid(func, grid):
     """More strips than CTAs: each CTA runs several strips in claim order (deadlock-free)."""
-    R, E, W = GEOMS[func][0]
+    R, E, W = GEOMS[func][0][:3]
     m, n = 32 * W * R * 5 + 17, 300
     a, b = _inputs(func, 5 + grid, m, n)
     _check(func, _run(func, R, E, W, a, b, grid_ctas=grid, reps=3), _ref(func, a, b))

@@ -30,8 +30,11 @@ def main():
     cfg = CONFIGS[args.cfg]
     pb = None
     for g in args.geoms:
-        R, E, W = (int(v) for v in g.split(","))
+        vals = [int(v) for v in g.split(",")]
+        R, E, W = vals[:3]
+        S = vals[3] if len(vals) > 3 else 0
         os.environ["LDDP_AD_R"], os.environ["LDDP_AD_E"], os.environ["LDDP_AD_W"] = str(R), str(E), str(W)
+        os.environ["LDDP_AD_S"] = str(S)
         if pb is None:
             pb = bench.build_problem(args.cfg, dev, lddp, 1, 0)
         else:

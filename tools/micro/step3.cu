@@ -256,6 +256,86 @@ void run_dual(const uint8_t* b, const uint8_t* a, int* out, long long* cyc, int 
   printf("DUAL R=%d E=%d: %.1f cycles/step (2 strips), %.2f cells/cycle/SMSP\n", R, E, s / n, 2.0 * 32 * R / (s / n));
 }
 
+
+// SPLIT: a lane's R rows as two sub-chains of R/2; the lower half runs one column behind the
+// upper half (its U at column c-1 was produced by the upper half one step earlier), so the two
+// chains of a step are independent: ILP 2 for one extra step of lane lag.
+template <int R, int E>
+__global__ void __launch_bounds__(128, 1) sweep_split(const uint8_t* __restrict__ b, int n, const uint8_t* __restrict__ a,
+                                                      int* out, long long* cyc) {
+  constexpr int H2 = R / 2;
+  __shared__ uint8_t sb[1 << 12];
+  __shared__ uint8_t mtab[4][64][32];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  for (int i = threadIdx.x; i < n && i < (1 << 12); i += blockDim.x) sb[i] = b[i];
+  for (int i = threadIdx.x; i < 4 * 64 * 32; i += blockDim.x) (&mtab[0][0][0])[i] = (uint8_t)(i * 37);
+  __syncthreads();
+  int hist[R], fifo[E + 1];
+  for (int r = 0; r < R; ++r) hist[r] = 0;
+  for (int d = 0; d <= E; ++d) fifo[d] = 0;
+  int mid = 0;      // upper half's last row at the previous step (U for the lower half)
+  int midUL = 0;    // ... two steps back (UL for the lower half)
+  int cprev = 0;    // previous step's match mask (the lower half's column)
+  const int one = n >> 30 | 1;
+  long long t0 = clock64();
+  for (int t = 0; t < n; t += 8) {
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      const int tt = t + u;
+      const int cc = (int)mtab[w][sb[(tt - lane * (E + 1)) & 4095] & 63][lane];
+      int UA = fifo[E - 1], ULA = fifo[E];
+      int UB = mid, ULB = midUL;
+      int nw[R];
+#pragma unroll
+      for (int r = 0; r < H2; ++r) {
+        {   // upper half, column c
+          const int L = hist[r];
+          const int t2 = ((cc >> r) & 1) ? ULA * one + one : ULA;
+          const int v = max(max(UA, L), t2);
+          ULA = L; UA = v; nw[r] = v;
+        }
+        {   // lower half, column c - 1
+          const int q = H2 + r;
+          const int L = hist[q];
+          const int t2 = ((cprev >> q) & 1) ? ULB * one + one : ULB;
+          const int v = max(max(UB, L), t2);
+          ULB = L; UB = v; nw[q] = v;
+        }
+      }
+      midUL = hist[H2 - 1];
+      mid = nw[H2 - 1];
+      cprev = cc;
+      const int rv = __shfl_sync(0xffffffffu, nw[R - 1], (lane + 31) & 31);
+#pragma unroll
+      for (int d = E; d > 0; --d) fifo[d] = fifo[d - 1];
+      fifo[0] = rv;
+#pragma unroll
+      for (int r = 0; r < R; ++r) hist[r] = nw[r];
+    }
+  }
+  long long t1 = clock64();
+  int acc = 0;
+  for (int r = 0; r < R; ++r) acc += hist[r];
+  for (int d = 0; d <= E; ++d) acc += fifo[d];
+  out[blockIdx.x * 128 + threadIdx.x] = acc;
+  if (lane == 0) cyc[blockIdx.x * 8 + w] = t1 - t0;
+}
+
+template <int R, int E>
+void run_split(const uint8_t* b, const uint8_t* a, int* out, long long* cyc, int n) {
+  sweep_split<R, E><<<148, 128>>>(b, n, a, out, cyc);
+  cudaDeviceSynchronize();
+  sweep_split<R, E><<<148, 128>>>(b, n, a, out, cyc);
+  cudaDeviceSynchronize();
+  long long h[148 * 8];
+  cudaMemcpy(h, cyc, sizeof(h), cudaMemcpyDeviceToHost);
+  double s = 0;
+  for (int i = 0; i < 148; ++i)
+    for (int w = 0; w < 4; ++w) s += (double)h[i * 8 + w];
+  s /= 148 * 4;
+  printf("SPLIT R=%d E=%d: %.1f cycles/step, %.2f cycles/cell\n", R, E, s / n, s / n / R);
+}
+
 int main() {
   const int n = 1 << 14;
   uint8_t *b, *a;
@@ -267,6 +347,10 @@ int main() {
   cudaMalloc(&cyc, 148 * 8 * 8);
   cudaMemset(b, 1, 1 << 16);
   cudaMemset(a, 1, 148 * 256 * 16);
+  run_split<6, 2>(b, a, out, cyc, n);
+  run_split<8, 2>(b, a, out, cyc, n);
+  run_split<12, 2>(b, a, out, cyc, n);
+  run_split<6, 1>(b, a, out, cyc, n);
   run_dual<6, 2>(b, a, out, cyc, n);
   run_dual<4, 2>(b, a, out, cyc, n);
   run_dual<3, 2>(b, a, out, cyc, n);
