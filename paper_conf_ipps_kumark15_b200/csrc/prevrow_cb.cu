@@ -27,6 +27,9 @@
 #include "cellfn.cuh"
 #include "params.h"
 #include "sync.cuh"
+#include <cuda.h>
+#include <cudaTypedefs.h>
+#include <cstring>
 
 namespace lddp {
 
@@ -54,6 +57,19 @@ __device__ __forceinline__ bool cb_bar_ready(uint32_t bar, uint32_t parity) {
       : "memory");
   return ok != 0;
 }
+// 2-D tensor TMA of one row group: box {EXT columns, kCbRG rows} at (x, y); out-of-table
+// elements (negative x, x >= W, y >= H) are zero-filled by the TMA unit.
+constexpr int kCbRG = 32;   // rows per tensor TMA
+constexpr int kCbNG = 3;    // row groups in flight per warp (ring = kCbNG * kCbRG rows)
+__device__ __forceinline__ void cb_tma_tile(uint32_t dst, const CUtensorMap* tmap, int x, int y, uint32_t bar,
+                                            uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.release.cta.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];" ::"r"(dst),
+      "l"(reinterpret_cast<uint64_t>(tmap)), "r"(x), "r"(y), "r"(bar)
+      : "memory");
+}
+
 // Bulk (TMA) row stream state of one warp: lane 0 issues one cp.async.bulk per row for the
 // in-table part of the warp's extended window; completion on one mbarrier per ring slot.
 struct CbBulk {
@@ -61,7 +77,8 @@ struct CbBulk {
   uint32_t bytes;     // in-table bytes of the window (multiple of 16)
   uint32_t bar0;      // shared address of slot 0's mbarrier
   const void* src0;   // global address of row 0's first in-table column
-  int irow, islot;    // next row to issue and its slot
+  int irow, islot;    // next row to issue and its slot (MODE 2: next row group's first row)
+  int x0;             // MODE 2: first column of the warp's window (may be negative)
   uint32_t cpar;      // phase parity of the slot being consumed
 };
 
@@ -75,8 +92,8 @@ __device__ __forceinline__ void cb_ld_pair2(const uint64_t* p, uint64_t& a, uint
 // One band of nr <= HB rows.  OUT: this lane holds out-of-table columns (their value is f's
 // boundary value in every row: one extra select per cell, taken only by the two edge blocks'
 // edge lanes -- warp-uniform for every other warp).
-template <class F, int VP, int D, bool TABLE, bool OUT, bool BULK>
-__device__ __forceinline__ void cb_band(CbBulk& bk, const int lane, const FillParams& p, typename F::T (&cur)[VP], typename F::GridT (&g)[VP],
+template <class F, int VP, int D, bool TABLE, bool OUT, int MODE>
+__device__ __forceinline__ void cb_band(CbBulk& bk, const CUtensorMap* tmap, const int lane, const FillParams& p, typename F::T (&cur)[VP], typename F::GridT (&g)[VP],
                                         const int nr, const int64_t r0,
                                         const typename F::GridT* ring, int& cslot, uint32_t& idst, int& ileft,
                                         int64_t& ioff, const int64_t pitch,
@@ -93,7 +110,9 @@ __device__ __forceinline__ void cb_band(CbBulk& bk, const int lane, const FillPa
     // The global address is formed into a fresh register from the lane's row-0 pointer and a
     // running element offset: updating the LDGSTS address register in place made the next row
     // wait on the copy's register read (long-scoreboard stalls on the pointer increment).
-    if constexpr (BULK) {
+    if constexpr (MODE == 2) {
+      // tensor rows arrive in groups of kCbRG: nothing to issue per row
+    } else if constexpr (MODE == 1) {
       if (lane == 0 && bk.irow < p.rows)
         cb_tma_row(bk.dst0 + bk.islot * EXT * 4, static_cast<const char*>(bk.src0) + (int64_t)bk.irow * pitch * 4,
                    bk.bytes, bk.bar0 + bk.islot * 8);
@@ -112,11 +131,28 @@ __device__ __forceinline__ void cb_band(CbBulk& bk, const int lane, const FillPa
     }
     G gn[VP];
     cslot = (cslot + 1 == D) ? 0 : cslot + 1;
-    if constexpr (BULK) {
+    if constexpr (MODE == 1) {
       if (cslot == 0) bk.cpar ^= 1u;
       if (r0 + r + 1 < p.rows)
         while (!cb_bar_ready(bk.bar0 + cslot * 8, bk.cpar)) {
         }
+    }
+    if constexpr (MODE == 2) {
+      if (cslot % kCbRG == 0) {
+        // entering a new row group: the previous group is fully read -> refill its slot with the
+        // group kCbNG ahead (one 2-D tensor TMA of kCbRG rows x EXT columns), then wait for this one
+        const int gnew = cslot / kCbRG;
+        const int gold = (gnew == 0 ? kCbNG : gnew) - 1;
+        if (cslot == 0) bk.cpar ^= 1u;
+        if (lane == 0) {
+          asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+          cb_tma_tile(bk.dst0 + gold * kCbRG * EXT * 4, tmap, bk.x0, bk.irow, bk.bar0 + gold * 8, kCbRG * EXT * 4);
+        }
+        bk.irow += kCbRG;
+        if (r0 + r + 1 < p.rows)
+          while (!cb_bar_ready(bk.bar0 + gnew * 8, bk.cpar)) {
+          }
+      }
     }
     const G* gs = ring + cslot * EXT;
 #pragma unroll
@@ -151,8 +187,10 @@ __device__ __forceinline__ void cb_band(CbBulk& bk, const int lane, const FillPa
   }
 }
 
-template <class F, int VP, int HB, int D, bool TABLE, bool BULK>
-__global__ void __launch_bounds__(256) prevrow_cb_kernel(const FillParams p) {
+template <class F, int VP, int HB, int D, bool TABLE, int MODE>
+__global__ void __launch_bounds__(256) prevrow_cb_kernel(const FillParams p, const __grid_constant__ CUtensorMap tmap_) {
+  const CUtensorMap* tmap = &tmap_;
+  static_assert(MODE != 2 || D == kCbNG * kCbRG, "tensor mode: ring = kCbNG groups of kCbRG rows");
   using T = typename F::T;
   using G = typename F::GridT;
   static_assert(!(F::kMask & NB_L), "prev-row category: f must not read L");
@@ -206,7 +244,24 @@ __global__ void __launch_bounds__(256) prevrow_cb_kernel(const FillParams p) {
     asm volatile("mov.b64 %0, %0;" : "+l"(pitch));   // held in a register, not reloaded per row
     int64_t ioff = 0;                                 // element offset of the next row to issue
     CbBulk bk{};
-    if constexpr (BULK) {
+    if constexpr (MODE == 2) {
+      const uint32_t wbase = smem_u32(reinterpret_cast<G*>(cb_smem) + (size_t)wl * D * EXT);
+      bk.dst0 = wbase;
+      bk.bar0 = smem_u32(reinterpret_cast<uint64_t*>(cb_smem + (size_t)nw * D * EXT * sizeof(G)) + wl * D);
+      bk.x0 = j0 - HB;
+      if (lane == 0) {
+        for (int k = 0; k < kCbNG; ++k)
+          asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bk.bar0 + 8 * k) : "memory");
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        for (int k = 0; k < kCbNG; ++k)
+          cb_tma_tile(wbase + k * kCbRG * EXT * 4, tmap, bk.x0, k * kCbRG, bk.bar0 + 8 * k, kCbRG * EXT * 4);
+      }
+      __syncwarp();
+      bk.irow = kCbNG * kCbRG;
+      bk.cpar = 0;
+      while (!cb_bar_ready(bk.bar0, 0u)) {
+      }
+    } else if constexpr (MODE == 1) {
       const uint32_t wbase = smem_u32(reinterpret_cast<G*>(cb_smem) + (size_t)wl * D * EXT);
       const int cs = max(j0 - HB, 0), ce = min(j0 - HB + EXT, W);
       bk.dst0 = wbase + (uint32_t)(cs - (j0 - HB)) * 4u;
@@ -267,9 +322,9 @@ __global__ void __launch_bounds__(256) prevrow_cb_kernel(const FillParams p) {
     for (int64_t r0 = 0; r0 < H; r0 += HB) {
       const int nr = (int)((H - r0 < HB) ? (H - r0) : HB);
       if (anyout)
-        cb_band<F, VP, D, TABLE, true, BULK>(bk, lane, p, cur, g, nr, r0, ring, cslot, idst, ileft, ioff, pitch, src, ssz, outv, omask, e0, j0, BW);
+        cb_band<F, VP, D, TABLE, true, MODE>(bk, tmap, lane, p, cur, g, nr, r0, ring, cslot, idst, ileft, ioff, pitch, src, ssz, outv, omask, e0, j0, BW);
       else
-        cb_band<F, VP, D, TABLE, false, BULK>(bk, lane, p, cur, g, nr, r0, ring, cslot, idst, ileft, ioff, pitch, src, ssz, outv, omask, e0, j0, BW);
+        cb_band<F, VP, D, TABLE, false, MODE>(bk, tmap, lane, p, cur, g, nr, r0, ring, cslot, idst, ileft, ioff, pitch, src, ssz, outv, omask, e0, j0, BW);
       if (r0 + HB >= H) break;   // last band: outputs below
       if (p.debug & 8) continue;   // development: no band exchange (wrong results; timing only)
       // ---- band boundary: publish own edges, take the neighbours' as halos
@@ -316,7 +371,7 @@ __global__ void __launch_bounds__(256) prevrow_cb_kernel(const FillParams p) {
         for (int v = 0; v < VP; ++v) cur[v] = (T)(uint32_t)pr[v];
       }
     }
-    if constexpr (!BULK) cp_async_wait_group<0>();
+    if constexpr (MODE == 0) cp_async_wait_group<0>();
 
     // ---- outputs of the last row
     T mn = INT_MAX;
@@ -351,11 +406,24 @@ __global__ void __launch_bounds__(256) prevrow_cb_kernel(const FillParams p) {
 
 // ---------------------------------------------------------------------------------------------
 // Compiled geometries: variant id -> (VP, HB, D); BW = 32*VP - 2*HB own columns per warp.
-template <class F, int VP, int HB, int D, bool BULK = false>
+// cuTensorMapEncodeTiled through the runtime's driver entry point (no libcuda link needed).
+static PFN_cuTensorMapEncodeTiled_v12000 cb_encode_fn() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  if (fn == nullptr) {
+    void* ptr = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &ptr, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(ptr);
+  }
+  return fn;
+}
+
+template <class F, int VP, int HB, int D, int MODE = 0>
 static cudaError_t cb_launch(const FillParams& p, int nw, bool query, int* out, cudaStream_t s) {
-  const size_t smem = (size_t)nw * D * 32 * VP * sizeof(typename F::GridT) + (BULK ? (size_t)nw * D * 8 : 0);
-  auto kt = prevrow_cb_kernel<F, VP, HB, D, true, BULK>;
-  auto kf = prevrow_cb_kernel<F, VP, HB, D, false, BULK>;
+  const size_t smem = (size_t)nw * D * 32 * VP * sizeof(typename F::GridT) + (MODE ? (size_t)nw * D * 8 : 0);
+  auto kt = prevrow_cb_kernel<F, VP, HB, D, true, MODE>;
+  auto kf = prevrow_cb_kernel<F, VP, HB, D, false, MODE>;
   cudaError_t e = cudaFuncSetAttribute(kt, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e == cudaSuccess) e = cudaFuncSetAttribute(kf, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
@@ -365,11 +433,26 @@ static cudaError_t cb_launch(const FillParams& p, int nw, bool query, int* out, 
     e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k, nw * 32, smem);
     out[0] = 32 * VP - 2 * HB;
     out[1] = occ;
+    if (MODE == 2 && cb_encode_fn() == nullptr) out[1] = 0;   // no tensor-map encoder: not usable
     return e;
+  }
+  CUtensorMap tm;
+  memset(&tm, 0, sizeof(tm));
+  if (MODE == 2) {   // the cost grid as a 2-D int32 tensor, box = kCbRG rows x the warp's window
+    PFN_cuTensorMapEncodeTiled_v12000 enc = cb_encode_fn();
+    if (enc == nullptr) return cudaErrorNotSupported;
+    const cuuint64_t dims[2] = {(cuuint64_t)p.cols, (cuuint64_t)p.rows};
+    const cuuint64_t strides[1] = {(cuuint64_t)p.grid_pitch * sizeof(typename F::GridT)};
+    const cuuint32_t box[2] = {(cuuint32_t)(32 * VP), (cuuint32_t)kCbRG};
+    const cuuint32_t estr[2] = {1, 1};
+    if (enc(&tm, CU_TENSOR_MAP_DATA_TYPE_INT32, 2, const_cast<void*>(p.grid), dims, strides, box, estr,
+            CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+      return cudaErrorInvalidValue;
   }
   const int grid = (p.nblocks + nw - 1) / nw;
   FillParams pp = p;
-  void* args[] = {&pp};
+  void* args[] = {&pp, &tm};
   return cudaLaunchCooperativeKernel((const void*)k, dim3(grid), dim3(nw * 32), args, smem, s);
 }
 
@@ -382,8 +465,10 @@ static cudaError_t cb_dispatch(int variant, const FillParams& p, int nw, bool qu
     case 3: return cb_launch<F, 16, 64, 32>(p, nw, query, out, s);
     case 4: return cb_launch<F, 8, 64, 96>(p, nw, query, out, s);
     case 5: return cb_launch<F, 4, 32, 64>(p, nw, query, out, s);   // BW 64
-    case 6: return cb_launch<F, 4, 32, 64, true>(p, nw, query, out, s);   // BW 64, TMA rows
-    case 7: return cb_launch<F, 8, 64, 48, true>(p, nw, query, out, s);   // BW 128, TMA rows
+    case 6: return cb_launch<F, 4, 32, 64, 1>(p, nw, query, out, s);   // BW 64, bulk TMA rows
+    case 7: return cb_launch<F, 8, 64, 48, 1>(p, nw, query, out, s);   // BW 128, bulk TMA rows
+    case 8: return cb_launch<F, 4, 32, 96, 2>(p, nw, query, out, s);   // BW 64, 2-D tensor TMA, 32-row groups
+    case 9: return cb_launch<F, 8, 64, 96, 2>(p, nw, query, out, s);   // BW 128, 2-D tensor TMA
     default: return cudaErrorInvalidValue;
   }
 }

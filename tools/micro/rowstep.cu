@@ -10,7 +10,7 @@
 #include <cstdint>
 #include <cuda_runtime.h>
 
-template <int VP, int MODE>
+template <int VP, int MODE, int RING = 16>
 __global__ void __launch_bounds__(128, 1) rows(int n, int* out, long long* cyc, const int* __restrict__ gsrc) {
   __shared__ __align__(16) int ring[4][8][32 * VP];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
@@ -19,16 +19,16 @@ __global__ void __launch_bounds__(128, 1) rows(int n, int* out, long long* cyc, 
   int cur[VP], gk[VP], gn[VP];
   for (int v = 0; v < VP; ++v) { cur[v] = lane + v; gk[v] = v; gn[v] = v; }
   // MODE 5 / 6: + one 16-byte cp.async per lane per row from global (6: every 4th row commits)
-  __shared__ __align__(16) int cring[4][16][32 * 4];
-  const uint32_t cbase = (uint32_t)__cvta_generic_to_shared(&cring[w][0][lane * 4]);
+  extern __shared__ __align__(16) int cdyn[];
+  const uint32_t cbase = (uint32_t)__cvta_generic_to_shared(cdyn + (size_t)w * RING * 128 + lane * 4);
   long long t0 = clock64();
   for (int r = 0; r < n; ++r) {
     if (MODE >= 5) {
       const int* src = gsrc + ((size_t)(r & 4095) * 32768 + blockIdx.x * 128 + threadIdx.x * 4);
-      asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(cbase + (r & 15) * 512), "l"(src) : "memory");
+      asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(cbase + (r & (RING - 1)) * 512), "l"(src) : "memory");
       if (MODE == 5 || (r & 3) == 3) {
         asm volatile("cp.async.commit_group;" ::: "memory");
-        asm volatile("cp.async.wait_group 14;" ::: "memory");
+        asm volatile("cp.async.wait_group %0;" ::"n"(RING - 2) : "memory");
       }
     }
     int g[VP];
@@ -69,18 +69,20 @@ __global__ void __launch_bounds__(128, 1) rows(int n, int* out, long long* cyc, 
   if (lane == 0) cyc[blockIdx.x * 4 + w] = t1 - t0;
 }
 
-template <int VP, int MODE>
+template <int VP, int MODE, int RING = 16>
 void run(int* out, long long* cyc, int n, const int* g) {
-  rows<VP, MODE><<<148, 128>>>(n, out, cyc, g);
+  const int dyn = 4 * RING * 512;
+  cudaFuncSetAttribute(rows<VP, MODE, RING>, cudaFuncAttributeMaxDynamicSharedMemorySize, dyn);
+  rows<VP, MODE, RING><<<148, 128, dyn>>>(n, out, cyc, g);
   cudaDeviceSynchronize();
-  rows<VP, MODE><<<148, 128>>>(n, out, cyc, g);
+  rows<VP, MODE, RING><<<148, 128, dyn>>>(n, out, cyc, g);
   cudaError_t e = cudaDeviceSynchronize();
   long long h[148 * 4];
   cudaMemcpy(h, cyc, sizeof(h), cudaMemcpyDeviceToHost);
   double s = 0;
   for (int i = 0; i < 148 * 4; ++i) s += (double)h[i];
   s /= 148 * 4;
-  printf("VP=%d MODE=%d: %.1f cycles/row (%s)\n", VP, MODE, s / n, cudaGetErrorString(e));
+  printf("VP=%d MODE=%d RING=%d: %.1f cycles/row (%s)\n", VP, MODE, RING, s / n, cudaGetErrorString(e));
 }
 
 int main() {
@@ -95,6 +97,7 @@ int main() {
   run<4, 1>(out, cyc, n, g);
   run<4, 4>(out, cyc, n, g);
   run<4, 5>(out, cyc, n, g);
-  run<4, 6>(out, cyc, n, g);
+  run<4, 5, 32>(out, cyc, n, g);
+  run<4, 5, 64>(out, cyc, n, g);
   return 0;
 }
