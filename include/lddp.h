@@ -186,6 +186,19 @@ lddp_status lddp_fill(lddp_plan_t plan, const lddp_inputs* in, const lddp_output
  * device->host and synchronises `stream`.  Device staging buffers are owned by the plan. */
 lddp_status lddp_fill_host(lddp_plan_t plan, const lddp_inputs* host_in,
                            const lddp_outputs* host_out, void* stream);
+/* Traceback of a LCS / Levenshtein / DTW table written by lddp_fill with
+ * LDDP_OUT_TABLE (same plan; T[i-1][j-1] = D[i][j], row / column 0 implied by f's boundary).
+ * One device thread walks from DP cell (m, n) towards the boundary and writes the visited cells
+ * (i, j), 1 <= i <= m, 1 <= j <= n, to path_i / path_j (device int32 arrays of capacity
+ * m + n, caller-owned) and their count to *path_len (device int64).  Rules (R14):
+ *   LCS   a_i == b_j -> diagonal; else up if D[i-1][j] >= D[i][j-1], else left (CLRS);
+ *   Lev   diagonal on a match with equal cost, else the first of substitution, deletion,
+ *         insertion that reproduces D[i][j];
+ *   DTW   argmin of (UL, U, L), ties in that order, ends at (1, 1).
+ * in->a / in->b: the fill's device inputs.  Enqueues on `stream`; errors: INVALID_ARG,
+ * UNSUPPORTED (another f), CUDA. */
+lddp_status lddp_traceback(lddp_plan_t plan, const lddp_inputs* in, const void* table, int64_t table_pitch,
+                           int32_t* path_i, int32_t* path_j, int64_t* path_len, void* stream);
 /* Synchronise `stream` and read the workspace's device status word (watchdog). */
 lddp_status lddp_status_check(lddp_plan_t plan, void* workspace, void* stream);
 

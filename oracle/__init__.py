@@ -147,3 +147,66 @@ def min2plus(init, c: int = 1, table: bool = False) -> Result:
 def diagmaxplus(init, c: int = 1, table: bool = False) -> Result:
     """Inverted-L synthetic f = max(init, UL) + c ([L298] §V.B)."""
     return _grid_fill(_L().oracle_diagmaxplus, init, (int(c),), table, want_col=True)
+
+
+def traceback(func: str, a, b, table):
+    """Traceback of a full oracle table (reading R14), plain Python loops: the DP cells
+    (i, j), 1-based, visited from (m, n) while i >= 1 and j >= 1.  ``table[i-1][j-1] = D[i][j]``;
+    row / column 0 are f's boundary.  LCS follows CLRS PRINT-LCS (match -> diagonal, else up when
+    D[i-1][j] >= D[i][j-1]); Levenshtein takes a free diagonal on a match, else the first of
+    substitution / deletion / insertion that reproduces D[i][j]; DTW the argmin of
+    (UL, U, L), ties in that order, ending at (1, 1)."""
+    m, n = len(a), len(b)
+    inf = float("inf")
+
+    def D(i, j):
+        if i >= 1 and j >= 1:
+            return table[i - 1][j - 1]
+        if func == "levenshtein":
+            return max(i, j)
+        if func == "dtw":
+            return 0.0 if i == 0 and j == 0 else inf
+        return 0
+
+    path = []
+    i, j = m, n
+    while i >= 1 and j >= 1:
+        path.append((i, j))
+        if func == "dtw":
+            if i == 1 and j == 1:
+                break
+            d, u, l = D(i - 1, j - 1), D(i - 1, j), D(i, j - 1)
+            if d <= u and d <= l:
+                i, j = i - 1, j - 1
+            elif u <= l:
+                i -= 1
+            else:
+                j -= 1
+        elif func == "lcs":
+            if a[i - 1] == b[j - 1]:
+                i, j = i - 1, j - 1
+            elif D(i - 1, j) >= D(i, j - 1):
+                i -= 1
+            else:
+                j -= 1
+        else:
+            here = D(i, j)
+            if a[i - 1] == b[j - 1] and here == D(i - 1, j - 1):
+                i, j = i - 1, j - 1
+            elif here == D(i - 1, j - 1) + 1:
+                i, j = i - 1, j - 1
+            elif here == D(i - 1, j) + 1:
+                i -= 1
+            else:
+                j -= 1
+    return path
+
+
+def lcs_string(a, b, path) -> bytes:
+    """The common subsequence a LCS traceback path spells (matched diagonal moves)."""
+    out = []
+    for k, (i, j) in enumerate(path):
+        nxt = path[k + 1] if k + 1 < len(path) else (i - 1, j - 1)
+        if nxt == (i - 1, j - 1) and a[i - 1] == b[j - 1]:
+            out.append(int(a[i - 1]))
+    return bytes(reversed(out))

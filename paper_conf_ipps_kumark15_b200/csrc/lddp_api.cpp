@@ -883,6 +883,28 @@ lddp_status lddp_comm_destroy(lddp_comm_t c) {
   return LDDP_OK;
 }
 
+lddp_status lddp_traceback(lddp_plan_t pl, const lddp_inputs* in, const void* table, int64_t table_pitch,
+                           int32_t* path_i, int32_t* path_j, int64_t* path_len, void* stream) {
+  try {
+    if (pl == nullptr || in == nullptr || table == nullptr || path_i == nullptr || path_j == nullptr ||
+        path_len == nullptr)
+      return fail(LDDP_ERR_INVALID_ARG, "NULL argument");
+    const lddp_desc& d = pl->desc;
+    if (d.func != LDDP_F_LCS && d.func != LDDP_F_LEVENSHTEIN && d.func != LDDP_F_DTW)
+      return fail(LDDP_ERR_UNSUPPORTED, "traceback: LCS, Levenshtein or DTW only (f=%d)", d.func);
+    if (table_pitch < d.cols) return fail(LDDP_ERR_INVALID_ARG, "table_pitch %lld < cols", (long long)table_pitch);
+    if ((d.rows > 0 && in->a == nullptr) || (d.cols > 0 && in->b == nullptr))
+      return fail(LDDP_ERR_INVALID_ARG, "traceback needs the fill's inputs a and b");
+    DeviceGuard dg(d.device);
+    cudaError_t e = lddp::launch_traceback(d.func, in->a, in->b, table, table_pitch, d.rows, d.cols, path_i, path_j,
+                                           path_len, (cudaStream_t)stream);
+    if (e != cudaSuccess) return cuda_fail(e, "traceback launch");
+    return LDDP_OK;
+  } catch (...) {
+    return fail(LDDP_ERR_INTERNAL, "exception in lddp_traceback");
+  }
+}
+
 lddp_status lddp_fill_multi(lddp_plan_t pl, const lddp_inputs* in, const lddp_outputs* out,
                             void* ws, lddp_comm_t c, void* stream) {
   try {

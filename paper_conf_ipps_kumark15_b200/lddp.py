@@ -83,6 +83,7 @@ _SIGS = {
     "lddp_comm_connect_local": (ctypes.c_int, [_P, _P]),
     "lddp_comm_destroy": (ctypes.c_int, [_P]),
     "lddp_fill_multi": (ctypes.c_int, [_P, ctypes.POINTER(lddp_inputs), ctypes.POINTER(lddp_outputs), _P, _P, _P]),
+    "lddp_traceback": (ctypes.c_int, [_P, ctypes.POINTER(lddp_inputs), _P, ctypes.c_int64, _P, _P, _P, _P]),
 }
 for _name, (_res, _args) in _SIGS.items():
     _fn = getattr(_lib, _name)
@@ -248,3 +249,18 @@ class Plan:
 
     def check(self, stream=None):
         lddp_status_check(self.handle, self.ws.data_ptr(), _stream_handle(stream))
+
+    def traceback(self, a, b, table, stream=None):
+        """Traceback of this plan's TABLE output (LCS / Levenshtein / DTW) on the device: returns
+        the visited DP cells (i, j), 1-based, from (m, n) backwards, as two int32 device tensors."""
+        import torch
+
+        cap = max(self.rows + self.cols, 1)
+        pi = torch.empty(cap, dtype=torch.int32, device=table.device)
+        pj = torch.empty(cap, dtype=torch.int32, device=table.device)
+        ln = torch.zeros(1, dtype=torch.int64, device=table.device)
+        inp = lddp_inputs(a=_ptr(a), b=_ptr(b), grid=None, grid_pitch=0)
+        _check(_lib.lddp_traceback(self.handle, ctypes.byref(inp), _ptr(table), table.stride(0), _ptr(pi), _ptr(pj),
+                                   _ptr(ln), _stream_handle(stream)), "lddp_traceback")
+        k = int(ln.item())
+        return pi[:k], pj[:k]

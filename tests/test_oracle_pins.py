@@ -459,3 +459,87 @@ def test_fig2_knight_grid():
                      ("Vertical", "vertical")]:
         vals = {SCHEDULES[pat](i, j, 6, 6) for i in range(6) for j in range(6)}
         assert len(vals) == counts[key], pat
+
+
+# ---------------------------------------------------------------------------------- traceback
+# Reading R14: the traceback rule of each sequence f.  Pinned by the textbook LCS
+# (CLRS Fig. 15.8 prints "BCBA" for X = ABCBDAB, Y = BDCABA with the up-on-ties rule) and by
+# properties any valid alignment must have, checked without the traceback code.
+
+def _is_subsequence(s, t):
+    it = iter(t)
+    return all(c in it for c in s)
+
+
+def _moves_ok(path, m, n):
+    if not path or path[0] != (m, n):
+        return False
+    for (i0, j0), (i1, j1) in zip(path, path[1:]):
+        if (i0 - i1, j0 - j1) not in ((1, 1), (1, 0), (0, 1)):
+            return False
+    return True
+
+
+def test_traceback_lcs_textbook(oracle_mod):
+    a, b = np.frombuffer(b"ABCBDAB", np.uint8), np.frombuffer(b"BDCABA", np.uint8)
+    r = oracle_mod.lcs(a, b, table=True)
+    path = oracle_mod.traceback("lcs", a, b, r.table)
+    assert oracle_mod.lcs_string(a, b, path) == b"BCBA"
+
+
+def test_traceback_lcs_random(oracle_mod):
+    rng = np.random.default_rng(3)
+    for _ in range(60):
+        m, n = rng.integers(1, 40, 2)
+        a = rng.integers(65, 69, m).astype(np.uint8)
+        b = rng.integers(65, 69, n).astype(np.uint8)
+        r = oracle_mod.lcs(a, b, table=True)
+        path = oracle_mod.traceback("lcs", a, b, r.table)
+        s = oracle_mod.lcs_string(a, b, path)
+        assert _moves_ok(path, m, n)
+        assert len(s) == r.score
+        assert _is_subsequence(s, bytes(a)) and _is_subsequence(s, bytes(b))
+
+
+def test_traceback_dtw_path_cost(oracle_mod):
+    """Integer-valued series: the path's summed |x - y| equals D(m, n) exactly; the path is a
+    warping path from (m, n) to (1, 1)."""
+    rng = np.random.default_rng(4)
+    for _ in range(60):
+        m, n = rng.integers(1, 30, 2)
+        x = rng.integers(-20, 21, m).astype(np.float32)
+        y = rng.integers(-20, 21, n).astype(np.float32)
+        r = oracle_mod.dtw(x, y, table=True)
+        path = oracle_mod.traceback("dtw", x, y, r.table)
+        assert _moves_ok(path, m, n) and path[-1] == (1, 1)
+        assert sum(abs(float(x[i - 1]) - float(y[j - 1])) for i, j in path) == float(r.score)
+
+
+def test_traceback_levenshtein_cost(oracle_mod):
+    """The alignment the path describes (diagonal: 0 / 1, vertical / horizontal: 1, then the
+    boundary tail) costs exactly the distance."""
+    rng = np.random.default_rng(5)
+    for _ in range(60):
+        m, n = rng.integers(1, 30, 2)
+        a = rng.integers(65, 69, m).astype(np.uint8)
+        b = rng.integers(65, 69, n).astype(np.uint8)
+        r = oracle_mod.levenshtein(a, b, table=True)
+        path = oracle_mod.traceback("levenshtein", a, b, r.table)
+        assert _moves_ok(path, m, n)
+        cost = 0
+        for k, (i, j) in enumerate(path):
+            if k + 1 < len(path):
+                i1, j1 = path[k + 1]
+            else:   # the move that leaves the table interior
+                i1, j1 = i - 1, j - 1
+                if not (i >= 1 and j >= 1):
+                    break
+                here = r.table[i - 1][j - 1]
+                diag = (max(i - 1, j - 1) if (i == 1 or j == 1) else r.table[i - 2][j - 2])
+                if not ((a[i - 1] == b[j - 1] and here == diag) or here == diag + 1):
+                    up = max(i - 1, j) if i == 1 else r.table[i - 2][j - 1]
+                    i1, j1 = (i - 1, j) if here == up + 1 else (i, j - 1)
+            cost += (int(a[i - 1] != b[j - 1]) if (i - i1, j - j1) == (1, 1) else 1)
+            if k + 1 == len(path):
+                cost += max(i1, j1)   # boundary tail: pure deletions / insertions
+        assert cost == r.score
