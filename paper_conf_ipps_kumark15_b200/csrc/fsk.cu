@@ -29,6 +29,11 @@ constexpr int kFsIn = 8;     // input chunks (16 B) per lane ring
 constexpr int kFsAhead = 6;  // chunks issued ahead of the lane's current chunk
 constexpr int kFsOut = 4;    // output chunks per lane ring
 
+// byte -> float without I2F (a quarter-rate XU op on the step's critical path): the byte as the
+// low mantissa bits of 2^23, minus 2^23 -- exact for 0..255, so bit-identical to (float)byte.
+__device__ __forceinline__ float fs_u8f(uint32_t byte) {
+  return __fsub_rn(__uint_as_float(0x4B000000u | byte), 8388608.0f);
+}
 __device__ __forceinline__ void fs_cp16(uint32_t dst, const void* src, uint32_t src_bytes) {
   asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src), "r"(src_bytes) : "memory");
 }
@@ -95,7 +100,7 @@ __global__ void __launch_bounds__(W * 32, 1) fsk_kernel(const FillParams p) {
 #pragma unroll
     for (int u = 0; u < 8; ++u) {
       const int c = -D + u - D * lane;
-      inq[u] = (float)inr[wid][lane][(c >> 4) & (kFsIn - 1)][c & 15];
+      inq[u] = fs_u8f(inr[wid][lane][(c >> 4) & (kFsIn - 1)][c & 15]);
     }
 
     // ---- links (the adiag protocol)
@@ -195,7 +200,7 @@ __global__ void __launch_bounds__(W * 32, 1) fsk_kernel(const FillParams p) {
 #pragma unroll
         for (int u = 0; u < 8; ++u) {
           const int cn = 32 * k - D + 8 * g + 8 + u - D * lane;
-          inn[u] = (float)inr[wid][lane][(cn >> 4) & (kFsIn - 1)][cn & 15];
+          inn[u] = fs_u8f(inr[wid][lane][(cn >> 4) & (kFsIn - 1)][cn & 15]);
         }
 #pragma unroll
         for (int u = 0; u < 8; ++u) {

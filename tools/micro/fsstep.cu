@@ -21,14 +21,22 @@ __global__ void __launch_bounds__(128, 1) fs(int n, int* out, long long* cyc) {
   float fifo[E + 3];
   for (int d = 0; d < E + 3; ++d) fifo[d] = 0.f;
   float eL = 0.f;
+  float inq[16];
+  for (int u = 0; u < 16; ++u) inq[u] = (float)inr[w][lane][(u - D * lane) & 127];
   long long t0 = clock64();
   for (int t = 0; t < n; t += 16) {
+    float inn[16];
+    if (MODE == 4) {
+#pragma unroll
+      for (int u = 0; u < 16; ++u) inn[u] = (float)inr[w][lane][(t + 16 + u - D * lane) & 127];
+    }
 #pragma unroll
     for (int u = 0; u < 16; ++u) {
       const int tau = t + u;
       const int c = tau - D * lane;
       float in;
-      if (MODE == 1) in = 100.f;
+      if (MODE == 4) in = inq[u];
+      else if (MODE == 1) in = 100.f;
       else if (MODE == 3) in = inf[w][lane][c & 63];
       else in = (float)inr[w][lane][c & 127];
       const float UR = MODE == 2 ? eL : fifo[E], U = MODE == 2 ? fifo[0] : fifo[E + 1], UL = fifo[E + 2];
@@ -46,6 +54,10 @@ __global__ void __launch_bounds__(128, 1) fs(int n, int* out, long long* cyc) {
 #pragma unroll
       for (int d = E + 2; d > 0; --d) fifo[d] = fifo[d - 1];
       fifo[0] = rv;
+    }
+    if (MODE == 4) {
+#pragma unroll
+      for (int u = 0; u < 16; ++u) inq[u] = inn[u];
     }
   }
   long long t1 = clock64();
@@ -77,6 +89,7 @@ int main() {
   run<1, 1>(out, cyc, n);
   run<1, 2>(out, cyc, n);
   run<1, 3>(out, cyc, n);
+  run<1, 4>(out, cyc, n);
   run<2, 0>(out, cyc, n);
   run<3, 0>(out, cyc, n);
   return 0;
