@@ -99,7 +99,8 @@ __device__ __forceinline__ void cb_band(CbBulk& bk, const CUtensorMap* tmap, con
                                         const typename F::GridT* ring, int& cslot, uint32_t& idst, int& ileft,
                                         int64_t& ioff, const int64_t pitch,
                                         const typename F::GridT* const (&src)[VP / 4], const uint32_t (&ssz)[VP / 4],
-                                        const typename F::T (&outv)[VP], const uint32_t omask, const int e0,
+                                        const typename F::T (&outv)[VP], const uint32_t omask, const bool lfix,
+                                        const int rfix, const int e0,
                                         const int j0, const int BW) {
   using T = typename F::T;
   using G = typename F::GridT;
@@ -162,17 +163,23 @@ __device__ __forceinline__ void cb_band(CbBulk& bk, const CUtensorMap* tmap, con
       gn[4 * s] = t.x; gn[4 * s + 1] = t.y; gn[4 * s + 2] = t.z; gn[4 * s + 3] = t.w;
     }
     const int64_t row = r0 + r;
-    const T lv = __shfl_up_sync(0xffffffffu, cur[VP - 1], 1);   // lane 0: own value (halo garbage)
+    T lv = __shfl_up_sync(0xffffffffu, cur[VP - 1], 1);   // lane 0: own value (halo garbage)
     const T rv = __shfl_down_sync(0xffffffffu, cur[0], 1);
+    // Table edges (OUT warps only): out-of-table cells are never forced; instead the two cells
+    // that read them take f's boundary value as that neighbour -- column 0's UL (always v = 0:
+    // e0 % 4 == 0) and column W-1's UR (v % 4 == 3 since W % 4 == 0).  Forcing every outside
+    // cell every row put selects on the row chain and made the two edge warps -- which pace all
+    // others through the halo exchange -- twice as slow as an interior warp.
+    if (OUT && lfix) lv = outv[0];
     T nw_[VP];
 #pragma unroll
     for (int v = 0; v < VP; ++v) {
       const T UL = (v > 0) ? cur[v - 1] : lv;
       const T U = cur[v];
-      const T UR = (v < VP - 1) ? cur[v + 1] : rv;
+      T UR = (v < VP - 1) ? cur[v + 1] : rv;
+      if (OUT && (v & 3) == 3) UR = (rfix == v) ? outv[VP - 1] : UR;
       typename F::OutT o;
       T x = F::f(U, UL, U, UR, typename F::RowCtx(0), typename F::ColCtx(0), g[v], row, e0 + v, p.param_c, o);
-      if (OUT) x = ((omask >> v) & 1u) ? outv[v] : x;
       nw_[v] = x;
       if (TABLE) {
         const int col = e0 + v;
@@ -227,6 +234,11 @@ __global__ void __launch_bounds__(256) prevrow_cb_kernel(const FillParams p, con
       outv[v] = col < 0 ? F::left(p, 0) : F::right(p, 0);
     }
     const bool anyout = __any_sync(0xffffffffu, omask != 0);
+    const bool lfix = (e0 == 0);                                         // column 0 at v = 0
+    const int rfix = (W - 1 >= e0 && W - 1 < e0 + VP) ? (W - 1 - e0) : -1;   // column W-1
+    T eoutv[VP];
+#pragma unroll
+    for (int v = 0; v < VP; ++v) eoutv[v] = (v == 0) ? F::left(p, 0) : F::right(p, 0);
     // 16-byte segments of this lane: all in or all out (W % 4 == 0, e0 % 4 == 0)
     uint32_t ssz[VP / 4];
     const G* src[VP / 4];
@@ -322,10 +334,16 @@ __global__ void __launch_bounds__(256) prevrow_cb_kernel(const FillParams p, con
 #pragma unroll 1
     for (int64_t r0 = 0; r0 < H; r0 += HB) {
       const int nr = (int)((H - r0 < HB) ? (H - r0) : HB);
+      // development trace (LDDP_TRACE): per band of block `trace_chunks`, clock64 at entry / exit
+      const bool trc = p.trace != nullptr && q == p.trace_chunks && lane == 0 && r0 / HB < 4096;
+      const long long tb0 = trc ? clock64() : 0;
       if (anyout)
-        cb_band<F, VP, D, TABLE, true, MODE>(bk, tmap, lane, p, cur, g, nr, r0, ring, cslot, idst, ileft, ioff, pitch, src, ssz, outv, omask, e0, j0, BW);
+        cb_band<F, VP, D, TABLE, true, MODE>(bk, tmap, lane, p, cur, g, nr, r0, ring, cslot, idst, ileft, ioff, pitch, src, ssz, eoutv, omask, lfix, rfix, e0, j0, BW);
       else
-        cb_band<F, VP, D, TABLE, false, MODE>(bk, tmap, lane, p, cur, g, nr, r0, ring, cslot, idst, ileft, ioff, pitch, src, ssz, outv, omask, e0, j0, BW);
+        cb_band<F, VP, D, TABLE, false, MODE>(bk, tmap, lane, p, cur, g, nr, r0, ring, cslot, idst, ileft, ioff, pitch, src, ssz, eoutv, omask, lfix, rfix, e0, j0, BW);
+      if (trc) {
+        p.trace[2 * (r0 / HB)] = (uint64_t)(clock64() - tb0);
+      }
       if (r0 + HB >= H) break;   // last band: outputs below
       if (p.debug & 8) continue;   // development: no band exchange (wrong results; timing only)
       // ---- band boundary: publish own edges, take the neighbours' as halos
@@ -371,6 +389,7 @@ __global__ void __launch_bounds__(256) prevrow_cb_kernel(const FillParams p, con
 #pragma unroll
         for (int v = 0; v < VP; ++v) cur[v] = (T)(uint32_t)pr[v];
       }
+      if (trc) p.trace[2 * (r0 / HB) + 1] = (uint64_t)(clock64() - tb0);
     }
     if constexpr (MODE == 0) cp_async_wait_group<0>();
 
