@@ -57,7 +57,9 @@ def main():
            "start_lag_ns_per_warp": float(np.diff(start.reshape(-1)).mean()),
            "last_end_ns": float(end.max()), "first_start_ns": [float(x) for x in start.reshape(-1)[:12]],
            "strip_start_ns": [float(x) for x in start[:8, 0]],
-           "end_ns_last_strip": [float(x) for x in end[-1]]}
+           "end_ns_last_strip": [float(x) for x in end[-1]],
+           "busy_cycles_per_step_by_warp": [float((busy[:, w]).mean() / steps) for w in range(W)],
+           "wait_top_frac_by_warp": [float(wt[:, w].sum() / cyc[:, w].sum()) for w in range(W)]}
     print(json.dumps(out, indent=1))
 
 
