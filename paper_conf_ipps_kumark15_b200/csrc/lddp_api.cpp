@@ -606,7 +606,7 @@ lddp_status lddp_plan(const lddp_desc* desc, lddp_plan_t* out) {
       // (16-byte cost segments; the row pitch / base alignment is checked per fill).
       pl->cb_variant = -1;
       const int cbv = env_int("LDDP_CB_VARIANT", 5);
-      const int cbnw = std::max(1, std::min(8, env_int("LDDP_CB_WARPS", 2)));
+      const int cbnw = std::max(1, std::min(8, env_int("LDDP_CB_WARPS", 4)));
       if (cbv >= 0 && d.cols > 0 && d.rows > 0 && d.cols % 4 == 0) {
         int q[2] = {0, 0};
         FillParams dummy{};

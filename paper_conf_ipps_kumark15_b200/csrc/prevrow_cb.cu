@@ -83,6 +83,35 @@ struct CbBulk {
   uint32_t cpar;      // phase parity of the slot being consumed
 };
 
+__device__ __forceinline__ void cb_cp8s(uint32_t dst, const void* src, uint32_t src_bytes) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;" ::"r"(dst), "l"(src), "r"(src_bytes) : "memory");
+}
+// lane segments: 16 bytes (4 columns) when VP % 4 == 0, else 8 bytes (2 columns)
+template <int VP> constexpr int kCbSeg = (VP % 4 == 0) ? 4 : 2;
+template <int VP> constexpr int kCbNSeg = VP / kCbSeg<VP>;
+template <int VP, class G>
+__device__ __forceinline__ void cb_issue(uint32_t idst, const G* const (&src)[kCbNSeg<VP>], const uint32_t (&ssz)[kCbNSeg<VP>],
+                                         int64_t ioff) {
+#pragma unroll
+  for (int s = 0; s < kCbNSeg<VP>; ++s) {
+    if constexpr (kCbSeg<VP> == 4) cb_cp16s(idst + 16 * s, src[s] + ioff, ssz[s]);
+    else cb_cp8s(idst + 8 * s, src[s] + ioff, ssz[s]);
+  }
+}
+template <int VP, class G>
+__device__ __forceinline__ void cb_lds(const G* gs, G (&g)[VP]) {
+#pragma unroll
+  for (int s = 0; s < kCbNSeg<VP>; ++s) {
+    if constexpr (kCbSeg<VP> == 4) {
+      const int4 t = *reinterpret_cast<const int4*>(gs + 4 * s);
+      g[4 * s] = t.x; g[4 * s + 1] = t.y; g[4 * s + 2] = t.z; g[4 * s + 3] = t.w;
+    } else {
+      const int2 t = *reinterpret_cast<const int2*>(gs + 2 * s);
+      g[2 * s] = t.x; g[2 * s + 1] = t.y;
+    }
+  }
+}
+
 __device__ __forceinline__ void cb_st_pair2(uint64_t* p, uint64_t a, uint64_t b) {
   asm volatile("st.relaxed.gpu.global.v2.u64 [%0], {%1, %2};" ::"l"(p), "l"(a), "l"(b) : "memory");
 }
@@ -98,7 +127,7 @@ __device__ __forceinline__ void cb_band(CbBulk& bk, const CUtensorMap* tmap, con
                                         const int nr, const int64_t r0,
                                         const typename F::GridT* ring, int& cslot, uint32_t& idst, int& ileft,
                                         int64_t& ioff, const int64_t pitch,
-                                        const typename F::GridT* const (&src)[VP / 4], const uint32_t (&ssz)[VP / 4],
+                                        const typename F::GridT* const (&src)[kCbNSeg<VP>], const uint32_t (&ssz)[kCbNSeg<VP>],
                                         const typename F::T (&outv)[VP], const uint32_t omask, const bool lfix,
                                         const int rfix, const int e0,
                                         const int j0, const int BW) {
@@ -121,10 +150,7 @@ __device__ __forceinline__ void cb_band(CbBulk& bk, const CUtensorMap* tmap, con
       ++bk.irow;
       bk.islot = (bk.islot + 1 == D) ? 0 : bk.islot + 1;
     } else {
-      if (ileft > 0) {
-#pragma unroll
-        for (int s = 0; s < VP / 4; ++s) cb_cp16s(idst + 16 * s, src[s] + ioff, ssz[s]);
-      }
+      if (ileft > 0) cb_issue<VP>(idst, src, ssz, ioff);
       ioff += pitch;
       --ileft;
       idst = (idst == iend) ? ibeg : idst + EXT * 4;
@@ -156,12 +182,7 @@ __device__ __forceinline__ void cb_band(CbBulk& bk, const CUtensorMap* tmap, con
           }
       }
     }
-    const G* gs = ring + cslot * EXT;
-#pragma unroll
-    for (int s = 0; s < VP / 4; ++s) {
-      const int4 t = *reinterpret_cast<const int4*>(gs + 4 * s);
-      gn[4 * s] = t.x; gn[4 * s + 1] = t.y; gn[4 * s + 2] = t.z; gn[4 * s + 3] = t.w;
-    }
+    cb_lds<VP>(ring + cslot * EXT, gn);
     const int64_t row = r0 + r;
     T lv = __shfl_up_sync(0xffffffffu, cur[VP - 1], 1);   // lane 0: own value (halo garbage)
     const T rv = __shfl_down_sync(0xffffffffu, cur[0], 1);
@@ -177,7 +198,7 @@ __device__ __forceinline__ void cb_band(CbBulk& bk, const CUtensorMap* tmap, con
       const T UL = (v > 0) ? cur[v - 1] : lv;
       const T U = cur[v];
       T UR = (v < VP - 1) ? cur[v + 1] : rv;
-      if (OUT && (v & 3) == 3) UR = (rfix == v) ? outv[VP - 1] : UR;
+      if (OUT && ((v & 3) == 3 || v == VP - 1)) UR = (rfix == v) ? outv[VP - 1] : UR;
       typename F::OutT o;
       T x = F::f(U, UL, U, UR, typename F::RowCtx(0), typename F::ColCtx(0), g[v], row, e0 + v, p.param_c, o);
       nw_[v] = x;
@@ -203,7 +224,7 @@ __global__ void __launch_bounds__(256) prevrow_cb_kernel(const FillParams p, con
   using G = typename F::GridT;
   static_assert(!(F::kMask & NB_L), "prev-row category: f must not read L");
   static_assert(sizeof(T) == 4 && sizeof(G) == 4, "32-bit cells and costs");
-  static_assert(VP % 4 == 0 && HB % VP == 0, "16-byte lane segments; halos made of whole lanes");
+  static_assert(VP % 2 == 0 && HB % VP == 0, "8- or 16-byte lane segments; halos made of whole lanes");
   constexpr int EXT = 32 * VP;
   constexpr int BW = EXT - 2 * HB;
   constexpr int HL = HB / VP;            // lanes per halo
@@ -240,13 +261,14 @@ __global__ void __launch_bounds__(256) prevrow_cb_kernel(const FillParams p, con
 #pragma unroll
     for (int v = 0; v < VP; ++v) eoutv[v] = (v == 0) ? F::left(p, 0) : F::right(p, 0);
     // 16-byte segments of this lane: all in or all out (W % 4 == 0, e0 % 4 == 0)
-    uint32_t ssz[VP / 4];
-    const G* src[VP / 4];
+    constexpr int SEG = kCbSeg<VP>;
+    uint32_t ssz[kCbNSeg<VP>];
+    const G* src[kCbNSeg<VP>];
 #pragma unroll
-    for (int s = 0; s < VP / 4; ++s) {
-      const int col = e0 + 4 * s;
+    for (int s = 0; s < kCbNSeg<VP>; ++s) {
+      const int col = e0 + SEG * s;
       const bool in = col >= 0 && col < W;
-      ssz[s] = in ? 16u : 0u;
+      ssz[s] = in ? 4u * SEG : 0u;
       asm volatile("mov.b32 %0, %0;" : "+r"(ssz[s]));   // opaque: no per-row rematerialisation
       src[s] = cost + (in ? col : 0);
     }
@@ -300,10 +322,7 @@ __global__ void __launch_bounds__(256) prevrow_cb_kernel(const FillParams p, con
     } else {
 #pragma unroll 1
       for (int k = 0; k < D - 1; ++k) {
-        if (ileft > 0) {
-#pragma unroll
-          for (int s = 0; s < VP / 4; ++s) cb_cp16s(idst + 16 * s, src[s] + ioff, ssz[s]);
-        }
+        if (ileft > 0) cb_issue<VP>(idst, src, ssz, ioff);
         ioff += pitch;
         --ileft;
         idst += EXT * 4;
@@ -314,11 +333,7 @@ __global__ void __launch_bounds__(256) prevrow_cb_kernel(const FillParams p, con
 
     // costs of row 0 (the band loop loads row r+1 while computing row r)
     G g[VP];
-#pragma unroll
-    for (int s = 0; s < VP / 4; ++s) {
-      const int4 t = *reinterpret_cast<const int4*>(ring + 4 * s);
-      g[4 * s] = t.x; g[4 * s + 1] = t.y; g[4 * s + 2] = t.z; g[4 * s + 3] = t.w;
-    }
+    cb_lds<VP>(ring, g);
 
     // row -1 (virtual): f's top initialisation
     T cur[VP];
@@ -745,6 +760,8 @@ static cudaError_t cb_dispatch(int variant, const FillParams& p, int nw, bool qu
     case 10: return gh_launch<F, 4, 32, 64, 4>(p, nw, query, out, s);  // BW 64, lane ghosts: SHFL every 4 rows
     case 11: return gh_launch<F, 8, 64, 48, 8>(p, nw, query, out, s);  // BW 128, lane ghosts every 8 rows
     case 12: return gh_launch<F, 8, 64, 48, 4>(p, nw, query, out, s);  // BW 128, lane ghosts every 4 rows
+    case 13: return cb_launch<F, 2, 16, 64>(p, nw, query, out, s);      // BW 32, 8-byte segments, 1024 warps for C4
+    case 14: return cb_launch<F, 2, 16, 96>(p, nw, query, out, s);      // BW 32, deeper ring
     default: return cudaErrorInvalidValue;
   }
 }
