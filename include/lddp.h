@@ -136,7 +136,13 @@ typedef struct {
     const void* grid;        /* FS: const uint8_t, MIN_PATH3/DIAG_MAXPLUS/MIN2_PLUS: const
                                 int32_t; rows x cols, row pitch grid_pitch elements             */
     int64_t grid_pitch;      /* elements; >= cols.  FS additionally needs pitch % 4 == 0 and a
-                                4-byte aligned base (word-wide pixel loads)                     */
+                                4-byte aligned base (word-wide pixel loads).  Fast paths, chosen
+                                per fill, fall back to the generic kernels otherwise:
+                                - FS (fsk.cu): cols % 16 == 0, grid and table pitches multiples
+                                  of 16 bytes, 16-byte aligned bases;
+                                - prev-row (prevrow_cb.cu): 32-bit grid, cols % 4 == 0, pitch
+                                  % 4 == 0, 16-byte aligned base, and the column blocks
+                                  co-resident on the device (checked at plan time)          */
 } lddp_inputs;
 
 typedef struct {
