@@ -39,17 +39,20 @@ __device__ __forceinline__ void fs_cp16(uint32_t dst, const void* src, uint32_t 
 }
 }  // namespace
 
-template <int W, int E>
+template <int W, int E, int R = 1>
 __global__ void __launch_bounds__(W * 32, 1) fsk_kernel(const FillParams p) {
-  constexpr int D = 2 + E;
-  constexpr int SH = W * 32;
+  // R rows per lane, skewed 2 columns apart inside the lane (independent pixels in a step);
+  // lane lag D = 2R + E; chunk step origin OFS = 2 + E (lane 31 injects top column tau + OFS)
+  constexpr int D = 2 * R + E;
+  constexpr int OFS = 2 + E;
+  constexpr int SH = W * 32 * R;
   using F = CellFS;
   __shared__ __align__(16) uint64_t ring[W][kAdRing][32];     // top stream of warp w >= 1
   __shared__ int cons[W];
   __shared__ __align__(16) float stg[W][32];                   // bottom staging row
   __shared__ __align__(16) float tstg[W][32];                  // top row of the current chunk
-  __shared__ __align__(16) uint8_t inr[W][32][kFsIn][16];      // per-lane input chunks
-  __shared__ __align__(16) uint8_t outr[W][32][kFsOut][16];    // per-lane output chunks
+  __shared__ __align__(16) uint8_t inr[W][32][R][kFsIn][16];   // per-(lane, row) input chunks
+  __shared__ __align__(16) uint8_t outr[W][32][R][kFsOut][16]; // per-(lane, row) output chunks
   __shared__ int strip_sh;
 
   Control* ctl = static_cast<Control*>(p.ctl);
@@ -77,31 +80,44 @@ __global__ void __launch_bounds__(W * 32, 1) fsk_kernel(const FillParams p) {
     __syncthreads();
     const int s = strip_sh;
     if (s >= p.nstrips) break;
-    const int64_t row = (int64_t)s * SH + wid * 32 + lane;
-    const bool rvalid = row < H;
-    const uint8_t* rin = img + (rvalid ? row : 0) * p.grid_pitch;
-    uint8_t* rout = out + (rvalid ? row : 0) * p.table_pitch;
-    const uint32_t inbase = smem_u32(&inr[wid][lane][0][0]);
+    const int64_t row0 = (int64_t)s * SH + (wid * 32 + lane) * R;
+    bool rvalid[R];
+    const uint8_t* rin[R];
+    uint8_t* rout[R];
+    uint32_t inbase[R];
+    int nq[R];
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      rvalid[r] = row0 + r < H;
+      rin[r] = img + (rvalid[r] ? row0 + r : 0) * p.grid_pitch;
+      rout[r] = out + (rvalid[r] ? row0 + r : 0) * p.table_pitch;
+      inbase[r] = smem_u32(&inr[wid][lane][r][0][0]);
+      nq[r] = (-OFS - D * lane - 2 * r) >> 4;   // floor(first column / 16)
+    }
     const uint32_t base = iter * (uint32_t)NQ + 1u;
 
-    // ---- input prologue: chunks q0 .. q0 + kFsAhead - 1 of this lane's first column
-    const int c_first = -D - D * lane;
-    int nq = c_first >> 4;   // floor(c / 16) (arithmetic shift)
-    for (int a = 0; a < kFsAhead; ++a, ++nq) {
-      const bool in = rvalid && nq >= 0 && 16 * nq < Wimg;
-      fs_cp16(inbase + (nq & (kFsIn - 1)) * 16, rin + (in ? 16 * nq : 0), in ? 16u : 0u);
+    // ---- input prologue: kFsAhead chunks per row from the row's first column
+    for (int a = 0; a < kFsAhead; ++a) {
+#pragma unroll
+      for (int r = 0; r < R; ++r) {
+        const bool in = rvalid[r] && nq[r] >= 0 && 16 * nq[r] < Wimg;
+        fs_cp16(inbase[r] + (nq[r] & (kFsIn - 1)) * 16, rin[r] + (in ? 16 * nq[r] : 0), in ? 16u : 0u);
+        ++nq[r];
+      }
       cp_async_commit();
     }
     cp_async_wait_group<kFsAhead - 4>();
     __syncwarp();
     // inputs of the first 8 steps (the step loop loads the NEXT group's inputs one group ahead:
     // LDS.U8 + I2F on the pixel chain cost ~40 cycles per step)
-    float inq[8];
+    float inq[R][8];
 #pragma unroll
-    for (int u = 0; u < 8; ++u) {
-      const int c = -D + u - D * lane;
-      inq[u] = fs_u8f(inr[wid][lane][(c >> 4) & (kFsIn - 1)][c & 15]);
-    }
+    for (int r = 0; r < R; ++r)
+#pragma unroll
+      for (int u = 0; u < 8; ++u) {
+        const int c = -OFS + u - D * lane - 2 * r;
+        inq[r][u] = fs_u8f(inr[wid][lane][r][(c >> 4) & (kFsIn - 1)][c & 15]);
+      }
 
     // ---- links (the adiag protocol)
     const int topsrc = (wid > 0) ? 1 : (s > 0 ? 2 : 0);
@@ -116,7 +132,9 @@ __global__ void __launch_bounds__(W * 32, 1) fsk_kernel(const FillParams p) {
     float fifo[E + 3];
 #pragma unroll
     for (int d = 0; d < E + 3; ++d) fifo[d] = 0.0f;
-    float eL = 0.0f;
+    float h[R][3];   // h[r][d]: row r's error at step tau-1-d (L of row r, UR/U/UL of row r+1)
+#pragma unroll
+    for (int r = 0; r < R; ++r) h[r][0] = h[r][1] = h[r][2] = 0.0f;
     bool ok = true;
 
     for (int k = 0; k < K && ok; ++k) {
@@ -186,11 +204,11 @@ __global__ void __launch_bounds__(W * 32, 1) fsk_kernel(const FillParams p) {
         injq[4] = a1.x; injq[5] = a1.y; injq[6] = a1.z; injq[7] = a1.w;
       }
 
-      // ---- 32 steps: tau = 32k - D + su (fully unrolled: the period test below is static)
+      // ---- 32 steps: tau = 32k - OFS + su (fully unrolled: the period test below is static)
 #pragma unroll
       for (int g = 0; g < 4; ++g) {
         float bv[8];
-        float inn[8], injn[8];
+        float inn[R][8], injn[8];
         if (g < 3) {
           const float4 a0 = reinterpret_cast<const float4*>(&tstg[wid][8 * g + 8])[0];
           const float4 a1 = reinterpret_cast<const float4*>(&tstg[wid][8 * g + 8])[1];
@@ -198,46 +216,63 @@ __global__ void __launch_bounds__(W * 32, 1) fsk_kernel(const FillParams p) {
           injn[4] = a1.x; injn[5] = a1.y; injn[6] = a1.z; injn[7] = a1.w;
         }
 #pragma unroll
-        for (int u = 0; u < 8; ++u) {
-          const int cn = 32 * k - D + 8 * g + 8 + u - D * lane;
-          inn[u] = fs_u8f(inr[wid][lane][(cn >> 4) & (kFsIn - 1)][cn & 15]);
-        }
+        for (int r = 0; r < R; ++r)
+#pragma unroll
+          for (int u = 0; u < 8; ++u) {
+            const int cn = 32 * k - OFS + 8 * g + 8 + u - D * lane - 2 * r;
+            inn[r][u] = fs_u8f(inr[wid][lane][r][(cn >> 4) & (kFsIn - 1)][cn & 15]);
+          }
 #pragma unroll
         for (int u = 0; u < 8; ++u) {
-          const int tau = 32 * k - D + 8 * g + u;
-          const int c = tau - D * lane;
-          const float in = inq[u];
-          const float UR = fifo[E], U = fifo[E + 1], UL = fifo[E + 2];
-          uint8_t o;
-          float e = F::f(eL, UL, U, UR, 0, 0, in, 0, 0, 0, o);
-          e = ((unsigned)c < (unsigned)Wimg) ? e : 0.0f;   // columns -1 and W are errors 0
-          outr[wid][lane][(c >> 4) & (kFsOut - 1)][c & 15] = o;
-          eL = e;
-          bv[u] = e;
+          const int tau = 32 * k - OFS + 8 * g + u;
+          float e[R];
+#pragma unroll
+          for (int r = 0; r < R; ++r) {
+            const int c = tau - D * lane - 2 * r;
+            const float UR = r == 0 ? fifo[E] : h[r - 1][0];
+            const float U = r == 0 ? fifo[E + 1] : h[r - 1][1];
+            const float UL = r == 0 ? fifo[E + 2] : h[r - 1][2];
+            uint8_t o;
+            float x = F::f(h[r][0], UL, U, UR, 0, 0, inq[r][u], 0, 0, 0, o);
+            e[r] = ((unsigned)c < (unsigned)Wimg) ? x : 0.0f;   // columns -1 and W are errors 0
+            outr[wid][lane][r][(c >> 4) & (kFsOut - 1)][c & 15] = o;
+          }
+#pragma unroll
+          for (int r = 0; r < R; ++r) {
+            h[r][2] = h[r][1];
+            h[r][1] = h[r][0];
+            h[r][0] = e[r];
+          }
+          bv[u] = e[R - 1];
           const float inj = injq[u];
-          const float sv = (lane == 31) ? inj : e;
+          const float sv = (lane == 31) ? inj : e[R - 1];
           const float rv = __shfl_sync(0xffffffffu, sv, (lane + 31) & 31);
 #pragma unroll
           for (int d = E + 2; d > 0; --d) fifo[d] = fifo[d - 1];
           fifo[0] = rv;
           if ((tau & 15) == 15) {
-            // period end: flush the completed output chunk, issue the next input chunk
-            const int qd = ((c + 1) >> 4) - 1;
-            if (rvalid && qd >= 0 && 16 * qd < Wimg) {
-              const uint4 w4 = *reinterpret_cast<const uint4*>(&outr[wid][lane][qd & (kFsOut - 1)][0]);
-              *reinterpret_cast<uint4*>(rout + 16 * qd) = w4;
+            // period end: per row, flush the completed output chunk and issue the next input chunk
+#pragma unroll
+            for (int r = 0; r < R; ++r) {
+              const int c = tau - D * lane - 2 * r;
+              const int qd = ((c + 1) >> 4) - 1;
+              if (rvalid[r] && qd >= 0 && 16 * qd < Wimg) {
+                const uint4 w4 = *reinterpret_cast<const uint4*>(&outr[wid][lane][r][qd & (kFsOut - 1)][0]);
+                *reinterpret_cast<uint4*>(rout[r] + 16 * qd) = w4;
+              }
+              const bool in2 = rvalid[r] && nq[r] >= 0 && 16 * nq[r] < Wimg;
+              fs_cp16(inbase[r] + (nq[r] & (kFsIn - 1)) * 16, rin[r] + (in2 ? 16 * nq[r] : 0), in2 ? 16u : 0u);
+              ++nq[r];
             }
-            const bool in2 = rvalid && nq >= 0 && 16 * nq < Wimg;
-            fs_cp16(inbase + (nq & (kFsIn - 1)) * 16, rin + (in2 ? 16 * nq : 0), in2 ? 16u : 0u);
             cp_async_commit();
-            ++nq;
             cp_async_wait_group<kFsAhead - 4>();
             __syncwarp();
           }
         }
 #pragma unroll
         for (int u = 0; u < 8; ++u) {
-          inq[u] = inn[u];
+#pragma unroll
+          for (int r = 0; r < R; ++r) inq[r][u] = inn[r][u];
           if (g < 3) injq[u] = injn[u];
         }
         if (lane == 31) {
@@ -283,14 +318,16 @@ __global__ void __launch_bounds__(W * 32, 1) fsk_kernel(const FillParams p) {
   }
 }
 
-// W warps per CTA (strip = 32 W rows), E = extra lane lag.  grid <= strips.
-cudaError_t launch_fsk(const FillParams& p, int W, int E, int grid, cudaStream_t s) {
-#define LDDP_FSK(w, e)                                                   \
-  if (W == w && E == e) {                                                \
-    fsk_kernel<w, e><<<grid, w * 32, 0, s>>>(p);                         \
+// W warps per CTA (strip = 32 W R rows), E = extra lane lag, R rows per lane.  grid <= strips.
+cudaError_t launch_fsk(const FillParams& p, int W, int E, int R, int grid, cudaStream_t s) {
+#define LDDP_FSK(w, e, r)                                                \
+  if (W == w && E == e && R == r) {                                      \
+    fsk_kernel<w, e, r><<<grid, w * 32, 0, s>>>(p);                      \
     return cudaGetLastError();                                           \
   }
-  LDDP_FSK(4, 0) LDDP_FSK(4, 1) LDDP_FSK(4, 2) LDDP_FSK(2, 0) LDDP_FSK(2, 1) LDDP_FSK(2, 2)
+  LDDP_FSK(4, 0, 1) LDDP_FSK(4, 1, 1) LDDP_FSK(4, 2, 1) LDDP_FSK(2, 0, 1) LDDP_FSK(2, 1, 1) LDDP_FSK(2, 2, 1)
+  LDDP_FSK(2, 0, 2) LDDP_FSK(2, 1, 2) LDDP_FSK(1, 0, 2) LDDP_FSK(1, 1, 2) LDDP_FSK(1, 2, 2) LDDP_FSK(1, 1, 1) LDDP_FSK(1, 0, 1) LDDP_FSK(1, 2, 1)
+  LDDP_FSK(1, 0, 3) LDDP_FSK(1, 1, 3) LDDP_FSK(1, 0, 4) LDDP_FSK(1, 1, 4)
 #undef LDDP_FSK
   return cudaErrorInvalidValue;
 }

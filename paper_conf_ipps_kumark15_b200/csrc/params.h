@@ -64,7 +64,7 @@ cudaError_t launch_prevrow(int func, const FillParams& p, int grid, cudaStream_t
 cudaError_t launch_prevrow_cb(int func, int variant, const FillParams& p, int nw, bool query, int* out,
                               cudaStream_t stream);
 // Floyd-Steinberg lane-systolic knight kernel (fsk.cu): W warps per CTA, E extra lane lag.
-cudaError_t launch_fsk(const FillParams& p, int W, int E, int grid, cudaStream_t stream);
+cudaError_t launch_fsk(const FillParams& p, int W, int E, int R, int grid, cudaStream_t stream);
 // Traceback of a LCS / Levenshtein / DTW table (traceback.cu): one thread, O(m + n).
 cudaError_t launch_traceback(int func, const void* a, const void* b, const void* table, int64_t pitch, int64_t m,
                              int64_t n, int32_t* pi, int32_t* pj, int64_t* len, cudaStream_t s);

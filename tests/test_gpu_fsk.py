@@ -20,11 +20,12 @@ FS_SHAPES = [(1, 16), (2, 32), (3, 16), (7, 48), (33, 64), (100, 160), (129, 256
 
 @pytest.fixture
 def fsk_env():
-    keys = ("LDDP_FSK", "LDDP_FSK_W", "LDDP_FSK_E")
+    keys = ("LDDP_FSK", "LDDP_FSK_W", "LDDP_FSK_E", "LDDP_FSK_R")
     old = {k: os.environ.get(k) for k in keys}
 
-    def set_(w, e, on=1):
+    def set_(w, e, on=1, r=1):
         os.environ["LDDP_FSK"], os.environ["LDDP_FSK_W"], os.environ["LDDP_FSK_E"] = str(on), str(w), str(e)
+        os.environ["LDDP_FSK_R"] = str(r)
 
     yield set_
     for k, v in old.items():
@@ -34,11 +35,12 @@ def fsk_env():
             os.environ[k] = v
 
 
-@pytest.mark.parametrize("w,e", [(4, 0), (4, 1), (4, 2), (2, 0), (2, 1), (2, 2)])
+@pytest.mark.parametrize("w,e,r", [(4, 0, 1), (4, 1, 1), (4, 2, 1), (2, 0, 1), (2, 1, 1), (2, 2, 1),
+                                   (2, 0, 2), (2, 1, 2), (1, 0, 2), (1, 1, 2), (1, 1, 1), (1, 0, 1), (1, 0, 3)])
 @pytest.mark.parametrize("shape", FS_SHAPES)
 @pytest.mark.parametrize("kind", ["ramp", "uniform"])
-def test_fsk_parity(fsk_env, w, e, shape, kind):
-    fsk_env(w, e)
+def test_fsk_parity(fsk_env, w, e, r, shape, kind):
+    fsk_env(w, e, r=r)
     H, W = shape
     img = inputs.gen_image(11 * H + W, H, W, kind)
     ref = oracle.fs(img)
