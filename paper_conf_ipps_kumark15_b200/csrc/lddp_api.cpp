@@ -519,6 +519,7 @@ lddp_status lddp_plan(const lddp_desc* desc, lddp_plan_t* out) {
         if (Wq > 0 && g.W != Wq) continue;
         if (Sq >= 0 && g.S != Sq) continue;
         if (Sq < 0 && g.S) continue;   // split geometries only on request: measured slower on B200 (C5 6.9 -> 11.6 ms)
+        if (Wq <= 0 && g.W < 4) continue;   // 1-2 warp CTAs only on request: measured slower (C5 7.3-8.2 ms)
         double c = ad_cost(d.func, g.R, g.E, g.W, g.S, d.rows, std::max<int64_t>(d.cols, 1), pl->sms);
         if (Rq > 0) c += 1e200 * std::abs(g.R - Rq);   // nearest compiled R to the request
         if (getenv("LDDP_PLAN_DEBUG"))
