@@ -115,6 +115,11 @@ struct AdWarp {
   CC* cring;        // this warp's column-context ring (shared memory)
   uint8_t* mtab;    // match cells: this warp's table mtab[c * 32 + lane] = rows r of the lane with
                     // a_r == c (bit r), c in [0, 256) (dynamic shared memory)
+  uint8_t* ctab;    // match cells, small alphabets: this warp's code table, byte c -> code 0..3 of
+                    // the warp's <= 4 distinct row characters, 4 for any other byte
+  uint32_t mpk;     // ... and this lane's masks packed by code (byte k = rows with code k)
+  bool small;       // warp-uniform: the warp's rows use <= 4 distinct characters -> the column
+                    // ring holds codes and a step's mask is one PRMT of mpk (no table lookup)
   int32_t one;      // run-time 1 held in a register (opaque to ptxas: no per-use constant loads)
   int64_t irow0;    // global row of this lane's row 0
 
@@ -226,7 +231,7 @@ struct AdWarp {
   // CHECKED: boundary columns -1 / n-1 (left values, right-column capture).
   // The 8-step body is identical for every warp role (no role branches inside it), so ptxas
   // can overlap consecutive steps and the body stays small for the instruction cache.
-  template <bool CHECKED>
+  template <bool CHECKED, bool SM>
   __device__ __forceinline__ void chunk(const FillParams& p, const int lane, const int k, T* stg, T* tstg) {
     const int n = p.cols;
     const int lane_off = lane * ELAG;
@@ -235,8 +240,10 @@ struct AdWarp {
     // warp's shared ring (the body reads it with LDS: lower latency than L1 hits)
     {
       const int slot = (32 * (k + 1) + lane) & (kAdCRing - 1);
-      cring[slot] = cpend;
-      if (slot < 8) cring[slot + kAdCRing] = cpend;
+      CC cv = cpend;
+      if constexpr (F::kMatchCells && SM) cv = CC(ctab[(uint32_t)cpend & 255u]);
+      cring[slot] = cv;
+      if (slot < 8) cring[slot + kAdCRing] = cv;
     }
     cpend = colctx_guard(p, 32 * (k + 2) + lane);
     // chunk k's top row -> shared memory; lane 31 takes its 8 injections per group from there,
@@ -259,7 +266,8 @@ struct AdWarp {
         const CC* cr = cring + ((tau0 + 8 - lane_off) & (kAdCRing - 1));
 #pragma unroll
         for (int u = 0; u < 8; ++u) {
-          if constexpr (F::kMatchCells) cnext[u] = CC(mtab[(uint32_t)cr[u] * 32 + lane]);
+          if constexpr (F::kMatchCells && SM) cnext[u] = CC(__byte_perm(mpk, 0u, (uint32_t)cr[u]));
+          else if constexpr (F::kMatchCells) cnext[u] = CC(mtab[(uint32_t)cr[u] * 32 + lane]);
           else cnext[u] = cr[u];
         }
       }
@@ -347,7 +355,7 @@ struct AdWarp {
     }
   }
 
-  template <bool CHECKED>
+  template <bool CHECKED, bool SM>
   __device__ __forceinline__ bool step_chunk(const FillParams& p, const int lane, const int k, const int NQ,
                                              const int TS, const int BS, Links& lk, Control* ctl) {
     // the staging row holds bottom chunk k-1-E (produced during chunk k-1): publish it first
@@ -355,12 +363,13 @@ struct AdWarp {
     if (!acquire_top(p, lane, k, NQ, TS, lk, ctl)) return false;
     // ring chunk k is in registers now: release its slot to warp w-1
     if (TS == 1 && k < NQ && lane == 0) ad_st_smem_i32(lk.cons_self, (int)(lk.base + (uint32_t)k));
-    chunk<CHECKED>(p, lane, k, lk.stg, lk.tstg);
+    chunk<CHECKED, SM>(p, lane, k, lk.stg, lk.tstg);
     return true;
   }
 
   // All K = NQ + E chunks of one strip: checked chunks at both ends, a tight steady loop between.
   // TS / BS are warp-uniform run-time roles handled at chunk granularity only.
+  template <bool SM>
   __device__ __forceinline__ bool strip(const FillParams& p, const int lane, const int NQ, const int TS,
                                         const int BS, Links& lk, Control* ctl) {
     const int n = p.cols;
@@ -370,11 +379,11 @@ struct AdWarp {
     int k1 = (n - 33 + E) >= 0 ? (n - 33 + E) / 32 + 1 : 0;
     k1 = max(k0, min(K, k1));
     for (int k = 0; k < k0; ++k)
-      if (!step_chunk<true>(p, lane, k, NQ, TS, BS, lk, ctl)) return false;
+      if (!step_chunk<true, SM>(p, lane, k, NQ, TS, BS, lk, ctl)) return false;
     for (int k = k0; k < k1; ++k)
-      if (!step_chunk<false>(p, lane, k, NQ, TS, BS, lk, ctl)) return false;
+      if (!step_chunk<false, SM>(p, lane, k, NQ, TS, BS, lk, ctl)) return false;
     for (int k = k1; k < K; ++k)
-      if (!step_chunk<true>(p, lane, k, NQ, TS, BS, lk, ctl)) return false;
+      if (!step_chunk<true, SM>(p, lane, k, NQ, TS, BS, lk, ctl)) return false;
     return publish_bottom(p, lane, K - 1 - ELAG, NQ, BS, lk, ctl);   // the last staged chunk
   }
 };
@@ -392,6 +401,7 @@ __global__ void __launch_bounds__(W * 32, 1) adiag_kernel(const FillParams p) {
   __shared__ int strip_sh;
   __shared__ int one_sh;
   extern __shared__ __align__(16) uint8_t ad_dyn_smem[];    // match tables (W x 256 x 32 u8)
+  __shared__ uint8_t ctab_sh[W][256];                       // per-warp small-alphabet code tables
 
   Control* ctl = static_cast<Control*>(p.ctl);
   const int lane = threadIdx.x & 31;
@@ -444,30 +454,75 @@ __global__ void __launch_bounds__(W * 32, 1) adiag_kernel(const FillParams p) {
     if (lane == 0) aw.fifo[0] = aw.leftval(p, wtop - 1);
     aw.cring = cring[wid];
     aw.one = ad_ld_smem_i32(&one_sh);   // a volatile load: ptxas cannot rematerialise it per use
+    aw.small = false;
+    if constexpr (F::kMatchCells) {
+      // Code table of the warp's row characters: if they take <= 4 distinct byte values (DNA),
+      // every step's match mask is one PRMT of a per-lane packed register instead of a table load.
+      aw.mtab = ad_dyn_smem + wid * 256 * 32;
+      aw.ctab = ctab_sh[wid];
+#pragma unroll
+      for (int j = 0; j < 8; ++j) aw.ctab[8 * lane + j] = 0xFF;
+      __syncwarp();
+#pragma unroll
+      for (int r = 0; r < R; ++r) {
+        const int c = (int)aw.rc[r];
+        if (c >= 0 && c < 256) aw.ctab[c] = 0;   // present (benign same-value races)
+      }
+      __syncwarp();
+      uint32_t pb = 0;
+#pragma unroll
+      for (int j = 0; j < 8; ++j) pb |= (aw.ctab[8 * lane + j] == 0 ? 1u : 0u) << j;
+      const int cnt = __popc(pb);
+      int pre = cnt;   // inclusive warp prefix sum of the distinct-character counts
+#pragma unroll
+      for (int off = 1; off < 32; off <<= 1) {
+        const int t = __shfl_up_sync(0xffffffffu, pre, off);
+        if (lane >= off) pre += t;
+      }
+      const int total = __shfl_sync(0xffffffffu, pre, 31);
+      aw.small = total <= 4;
+      __syncwarp();
+      if (aw.small) {
+        const int base0 = pre - cnt;
+#pragma unroll
+        for (int j = 0; j < 8; ++j)
+          aw.ctab[8 * lane + j] = ((pb >> j) & 1u) ? (uint8_t)(base0 + __popc(pb & ((1u << j) - 1u))) : (uint8_t)4;
+        __syncwarp();
+        aw.mpk = 0;
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+          const int c = (int)aw.rc[r];
+          if (c >= 0 && c < 256) aw.mpk |= 1u << (8 * aw.ctab[c] + r);
+        }
+      } else {
+        // this warp's match table for its lanes' rows (virtual rows match nothing)
+        for (int c = 0; c < 256; ++c) aw.mtab[c * 32 + lane] = 0;
+        __syncwarp();
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+          const int c = (int)aw.rc[r];
+          if (c >= 0 && c < 256) aw.mtab[c * 32 + lane] |= (uint8_t)(1u << r);
+        }
+      }
+      __syncwarp();
+    }
     for (int q = -E - 1 - S; q <= 0; ++q) {
       const int slot = (32 * q + lane) & (kAdCRing - 1);
-      const typename F::ColCtx v = aw.colctx_guard(p, 32 * q + lane);
+      typename F::ColCtx v = aw.colctx_guard(p, 32 * q + lane);
+      if constexpr (F::kMatchCells) {
+        if (aw.small) v = typename F::ColCtx(aw.ctab[(uint32_t)v & 255u]);
+      }
       aw.cring[slot] = v;
       if (slot < 8) aw.cring[slot + kAdCRing] = v;
     }
     aw.cpend = aw.colctx_guard(p, 32 + lane);
     __syncwarp();
-    if constexpr (F::kMatchCells) {
-      // this warp's match table for its lanes' rows (virtual rows match nothing)
-      aw.mtab = ad_dyn_smem + wid * 256 * 32;
-      for (int c = 0; c < 256; ++c) aw.mtab[c * 32 + lane] = 0;
-      __syncwarp();
-#pragma unroll
-      for (int r = 0; r < R; ++r) {
-        const int c = (int)aw.rc[r];
-        if (c >= 0 && c < 256) aw.mtab[c * 32 + lane] |= (uint8_t)(1u << r);
-      }
-      __syncwarp();
-    }
 #pragma unroll
     for (int u = 0; u < 8; ++u) {
       const typename F::ColCtx c = aw.cring[((-E - lane * AW::ELAG) & (kAdCRing - 1)) + u];
-      if constexpr (F::kMatchCells) aw.ccur[u] = typename F::ColCtx(aw.mtab[(uint32_t)c * 32 + lane]);
+      if constexpr (F::kMatchCells)
+        aw.ccur[u] = aw.small ? typename F::ColCtx(__byte_perm(aw.mpk, 0u, (uint32_t)c))
+                              : typename F::ColCtx(aw.mtab[(uint32_t)c * 32 + lane]);
       else aw.ccur[u] = c;
     }
 
@@ -502,7 +557,11 @@ __global__ void __launch_bounds__(W * 32, 1) adiag_kernel(const FillParams p) {
     lk.wait_bp = 0;
     aw.tp = 0;
     if (topsrc == 2) aw.tq1 = ad_ld_gpu(lk.gprev + lane);
-    ok = ok && aw.strip(p, lane, NQ, topsrc, botsnk, lk, ctl);
+    if constexpr (F::kMatchCells)
+      ok = ok && (aw.small ? aw.template strip<true>(p, lane, NQ, topsrc, botsnk, lk, ctl)
+                           : aw.template strip<false>(p, lane, NQ, topsrc, botsnk, lk, ctl));
+    else
+      ok = ok && aw.template strip<false>(p, lane, NQ, topsrc, botsnk, lk, ctl);
     const long long wait_bp = lk.wait_bp;
     if (p.trace != nullptr && lane == 0) {   // per (strip, warp): start, end, cycles, waits
       uint64_t* tr = p.trace + ((int64_t)s * W + wid) * 6;

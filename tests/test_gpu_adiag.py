@@ -97,3 +97,27 @@ def test_adiag_large(func):
     got = run_gpu(func, "anti_diagonal", a=a, b=b, outputs=("score", "last_row", "last_col"), reps=2)
     assert '"adiag"' in got["plan"]
     _check(func, got, _ref(func, a, b))
+
+
+@pytest.mark.parametrize("func", ["lcs", "levenshtein"])
+@pytest.mark.parametrize("alphabet", ["bytes", "mixed", "ascii26"])
+@pytest.mark.parametrize("shape", [(700, 900), (3001, 517)])
+def test_adiag_alphabets(func, alphabet, shape):
+    """Match cells take two paths per warp: <= 4 distinct row characters (DNA: a per-lane packed
+    mask register, one PRMT per step) or the per-warp 256-entry match table.  Cover both and warps
+    of both kinds in one fill."""
+    m, n = shape
+    rng = np.random.default_rng(m + 3 * n)
+    if alphabet == "bytes":
+        a = rng.integers(0, 256, m, dtype=np.uint8)
+        b = rng.integers(0, 256, n, dtype=np.uint8)
+    elif alphabet == "ascii26":
+        a = rng.integers(65, 91, m).astype(np.uint8)
+        b = rng.integers(65, 91, n).astype(np.uint8)
+    else:   # first half DNA (small-alphabet warps), second half wide (table warps)
+        a = np.concatenate([np.frombuffer(b"ACGT", np.uint8)[rng.integers(0, 4, m // 2)],
+                            rng.integers(60, 80, m - m // 2).astype(np.uint8)])
+        b = np.concatenate([np.frombuffer(b"ACGT", np.uint8)[rng.integers(0, 4, n // 2)],
+                            rng.integers(60, 80, n - n // 2).astype(np.uint8)])
+    got = run_gpu(func, "anti_diagonal", a=a, b=b, outputs=("score", "last_row", "last_col"))
+    _check(func, got, _ref(func, a, b))
