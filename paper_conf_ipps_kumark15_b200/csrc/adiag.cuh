@@ -118,6 +118,8 @@ struct AdWarp {
   uint8_t* ctab;    // match cells, small alphabets: this warp's code table, byte c -> code 0..3 of
                     // the warp's <= 4 distinct row characters, 4 for any other byte
   uint32_t mpk;     // ... and this lane's masks packed by code (byte k = rows with code k)
+  uint32_t* cnib;   // small alphabets: the warp's column codes, 4 bits per column, 8 per word
+                    // (32 words for the 256-column ring + 1 mirrored word for the funnel read)
   bool small;       // warp-uniform: the warp's rows use <= 4 distinct characters -> the column
                     // ring holds codes and a step's mask is one PRMT of mpk (no table lookup)
   int32_t one;      // run-time 1 held in a register (opaque to ptxas: no per-use constant loads)
@@ -240,10 +242,20 @@ struct AdWarp {
     // warp's shared ring (the body reads it with LDS: lower latency than L1 hits)
     {
       const int slot = (32 * (k + 1) + lane) & (kAdCRing - 1);
-      CC cv = cpend;
-      if constexpr (F::kMatchCells && SM) cv = CC(ctab[(uint32_t)cpend & 255u]);
-      cring[slot] = cv;
-      if (slot < 8) cring[slot + kAdCRing] = cv;
+      if constexpr (F::kMatchCells && SM) {
+        // 8 lanes' codes -> one word of nibbles (column slot 8w + j at bits 4j)
+        uint32_t v = (uint32_t)ctab[(uint32_t)cpend & 255u] << (4 * (lane & 7));
+        v |= __shfl_xor_sync(0xffffffffu, v, 1);
+        v |= __shfl_xor_sync(0xffffffffu, v, 2);
+        v |= __shfl_xor_sync(0xffffffffu, v, 4);
+        if ((lane & 7) == 0) {
+          cnib[slot >> 3] = v;
+          if (slot == 0) cnib[kAdCRing / 8] = v;
+        }
+      } else {
+        cring[slot] = cpend;
+        if (slot < 8) cring[slot + kAdCRing] = cpend;
+      }
     }
     cpend = colctx_guard(p, 32 * (k + 2) + lane);
     // chunk k's top row -> shared memory; lane 31 takes its 8 injections per group from there,
@@ -262,12 +274,20 @@ struct AdWarp {
     for (int g = 0; g < 4; ++g) {
       CC cnext[8];
       const int tau0 = 32 * k - E + 8 * g;
-      {
+      if constexpr (F::kMatchCells && SM) {
+        // the next group's 8 column codes (one funnel shift of two words), then two PRMTs give
+        // the 8 steps' match masks (code 4 selects a zero byte: matches nothing)
+        const int cn = (tau0 + 8 - lane_off) & (kAdCRing - 1);
+        const uint32_t codes = __funnelshift_r(cnib[cn >> 3], cnib[(cn >> 3) + 1], 4 * (cn & 7));
+        const uint32_t m0 = __byte_perm(mpk, 0u, codes);
+        const uint32_t m1 = __byte_perm(mpk, 0u, codes >> 16);
+#pragma unroll
+        for (int u = 0; u < 8; ++u) cnext[u] = CC((u < 4 ? m0 : m1) >> (8 * (u & 3)));
+      } else {
         const CC* cr = cring + ((tau0 + 8 - lane_off) & (kAdCRing - 1));
 #pragma unroll
         for (int u = 0; u < 8; ++u) {
-          if constexpr (F::kMatchCells && SM) cnext[u] = CC(__byte_perm(mpk, 0u, (uint32_t)cr[u]));
-          else if constexpr (F::kMatchCells) cnext[u] = CC(mtab[(uint32_t)cr[u] * 32 + lane]);
+          if constexpr (F::kMatchCells) cnext[u] = CC(mtab[(uint32_t)cr[u] * 32 + lane]);
           else cnext[u] = cr[u];
         }
       }
@@ -402,6 +422,7 @@ __global__ void __launch_bounds__(W * 32, 1) adiag_kernel(const FillParams p) {
   __shared__ int one_sh;
   extern __shared__ __align__(16) uint8_t ad_dyn_smem[];    // match tables (W x 256 x 32 u8)
   __shared__ uint8_t ctab_sh[W][256];                       // per-warp small-alphabet code tables
+  __shared__ uint32_t cnib_sh[W][kAdCRing / 8 + 1];         // per-warp column codes (nibbles)
 
   Control* ctl = static_cast<Control*>(p.ctl);
   const int lane = threadIdx.x & 31;
@@ -506,11 +527,21 @@ __global__ void __launch_bounds__(W * 32, 1) adiag_kernel(const FillParams p) {
       }
       __syncwarp();
     }
+    aw.cnib = cnib_sh[wid];
     for (int q = -E - 1 - S; q <= 0; ++q) {
       const int slot = (32 * q + lane) & (kAdCRing - 1);
       typename F::ColCtx v = aw.colctx_guard(p, 32 * q + lane);
       if constexpr (F::kMatchCells) {
-        if (aw.small) v = typename F::ColCtx(aw.ctab[(uint32_t)v & 255u]);
+        if (aw.small) {
+          uint32_t w = (uint32_t)aw.ctab[(uint32_t)v & 255u] << (4 * (lane & 7));
+          w |= __shfl_xor_sync(0xffffffffu, w, 1);
+          w |= __shfl_xor_sync(0xffffffffu, w, 2);
+          w |= __shfl_xor_sync(0xffffffffu, w, 4);
+          if ((lane & 7) == 0) {
+            aw.cnib[slot >> 3] = w;
+            if (slot == 0) aw.cnib[kAdCRing / 8] = w;
+          }
+        }
       }
       aw.cring[slot] = v;
       if (slot < 8) aw.cring[slot + kAdCRing] = v;
@@ -521,7 +552,7 @@ __global__ void __launch_bounds__(W * 32, 1) adiag_kernel(const FillParams p) {
     for (int u = 0; u < 8; ++u) {
       const typename F::ColCtx c = aw.cring[((-E - lane * AW::ELAG) & (kAdCRing - 1)) + u];
       if constexpr (F::kMatchCells)
-        aw.ccur[u] = aw.small ? typename F::ColCtx(__byte_perm(aw.mpk, 0u, (uint32_t)c))
+        aw.ccur[u] = aw.small ? typename F::ColCtx(__byte_perm(aw.mpk, 0u, (uint32_t)aw.ctab[(uint32_t)c & 255u]))
                               : typename F::ColCtx(aw.mtab[(uint32_t)c * 32 + lane]);
       else aw.ccur[u] = c;
     }
