@@ -198,7 +198,7 @@ __device__ __forceinline__ void cb_band(CbBulk& bk, const CUtensorMap* tmap, con
       const T UL = (v > 0) ? cur[v - 1] : lv;
       const T U = cur[v];
       T UR = (v < VP - 1) ? cur[v + 1] : rv;
-      if (OUT && ((v & 3) == 3 || v == VP - 1)) UR = (rfix == v) ? outv[VP - 1] : UR;
+      if (OUT && (VP % 4 != 0 || (v & 3) == 3)) UR = (rfix == v) ? outv[VP - 1] : UR;
       typename F::OutT o;
       T x = F::f(U, UL, U, UR, typename F::RowCtx(0), typename F::ColCtx(0), g[v], row, e0 + v, p.param_c, o);
       nw_[v] = x;
@@ -762,6 +762,8 @@ static cudaError_t cb_dispatch(int variant, const FillParams& p, int nw, bool qu
     case 12: return gh_launch<F, 8, 64, 48, 4>(p, nw, query, out, s);  // BW 128, lane ghosts every 4 rows
     case 13: return cb_launch<F, 2, 16, 64>(p, nw, query, out, s);      // BW 32, 8-byte segments, 1024 warps for C4
     case 14: return cb_launch<F, 2, 16, 96>(p, nw, query, out, s);      // BW 32, deeper ring
+    case 17: return cb_launch<F, 6, 48, 48>(p, nw, query, out, s);      // BW 96, exchange every 48 rows
+    case 18: return cb_launch<F, 6, 48, 32>(p, nw, query, out, s);      // BW 96, 32-row ring
     default: return cudaErrorInvalidValue;
   }
 }

@@ -36,7 +36,7 @@ def cb_env():
             os.environ[k] = v
 
 
-@pytest.mark.parametrize("variant,warps", [(0, 2), (1, 1), (2, 2), (3, 1), (4, 2), (0, 4), (5, 4), (5, 2), (6, 2), (6, 4), (7, 2), (7, 1), (8, 2), (8, 1), (8, 4), (9, 2), (10, 2), (10, 1), (10, 4), (11, 2), (12, 2), (13, 2), (13, 4), (13, 8), (14, 4)])
+@pytest.mark.parametrize("variant,warps", [(0, 2), (1, 1), (2, 2), (3, 1), (4, 2), (0, 4), (5, 4), (5, 2), (6, 2), (6, 4), (7, 2), (7, 1), (8, 2), (8, 1), (8, 4), (9, 2), (10, 2), (10, 1), (10, 4), (11, 2), (12, 2), (13, 2), (13, 4), (13, 8), (14, 4), (17, 4), (17, 2), (18, 4)])
 @pytest.mark.parametrize("shape", CB_SHAPES)
 def test_minpath3_cb(cb_env, variant, warps, shape):
     cb_env(variant, warps)
