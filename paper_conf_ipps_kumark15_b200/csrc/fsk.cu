@@ -3,18 +3,22 @@
 // §VI.B [L341] with the dependency constraint [L343-L344]).  The default FS kernel when the image
 // width and row pitch are multiples of 16 bytes (wavefront.cuh is the fallback).
 //
-//  * STRIPS of SH = 32*W rows (top-aligned; rows >= H are computed but never stored).  A CTA of W
-//    warps claims strips in increasing order; lane k of warp w owns ONE row i and processes
-//    column c = tau - D*k at warp step tau, D = 2 + E: the knight-move skew of 2 columns per row
-//    plus E steps of slack for the rotate SHFL that carries the error row to the lane below.
-//  * Lane k receives e(i-1, .) from lane k-1 through that one SHFL per step into a register FIFO:
-//    UR = fifo[E], U = fifo[E+1], UL = fifo[E+2]; L is the lane's own previous error.  Lane 31
-//    injects the warp's top row (the previous warp's bottom row) into the same SHFL.
+//  * STRIPS of SH = 32*W*R rows (top-aligned; rows >= H are computed but never stored).  A CTA of
+//    W warps claims strips in increasing order; lane k of warp w owns R rows and processes column
+//    c = tau - D*k - 2r for its row r at warp step tau, D = 2R + E: the knight-move skew of 2
+//    columns per row plus E steps of slack for the rotate SHFL that carries the lane's last
+//    row to the lane below.  Rows r >= 1 take UR / U / UL from row r-1's 3-step error history.
+//    Default W = 1, R = 1, E = 1 (measured best: every handoff through global boundary rows).
+//  * Row 0 of lane k receives e(i-1, .) from lane k-1 through that one SHFL per step into a
+//    register FIFO: UR = fifo[E], U = fifo[E+1], UL = fifo[E+2]; L is the row's previous error.
+//    Lane 31 injects the warp's top row (the previous warp's bottom row) into the same SHFL, its
+//    8 values per group loaded from shared memory one group ahead.
 //  * Pixel arithmetic = CellFS::f, the oracle's pull form and operation order
 //    ((((in + e_UL/16) + e_U*5/16) + e_UR*3/16) + e_L*7/16, threshold 128, e = v - out), built
 //    with --fmad=false: bit-exact.  Absent neighbours are errors of +0 (v + (+0) == v exactly).
-//  * Image rows stream through a per-lane shared ring of 16-byte chunks (cp.async, 6 chunks
-//    ahead); output bytes are collected in a per-lane 4-chunk ring and stored 16 bytes at a time.
+//  * Image rows stream through a per-(lane, row) shared ring of 16-byte chunks (cp.async, 6 chunks
+//    ahead), read one 8-step group ahead and converted by mantissa insertion (no I2F); output
+//    bytes are collected in a per-row 4-chunk ring and stored 16 bytes at a time.
 //  * Warp and strip handoffs of the error rows are the adiag protocol (adiag.cuh): tagged
 //    (value, tag) pairs in a shared ring (warp w -> w+1) or in global memory (strip s -> s+1),
 //    validated per 32-column chunk; no flags, no fences.

@@ -18,10 +18,14 @@
 //  * Edge exchange = (value, tag) 64-bit pairs in global memory (single-copy atomic): the
 //    consumer polls the data itself, no flag, no fence.  Tag = hash(fill epoch) + band.
 //  * Cost rows (the HBM stream, 4 B/cell) flow through a per-warp D-row shared-memory ring
-//    filled by 16-byte cp.async (LDGSTS.128, L1 bypass), D-1 rows ahead of the row being
-//    computed; every lane copies exactly the columns it later reads, so the ring needs no warp
-//    synchronisation at all.
+//    filled by 16-byte cp.async (LDGSTS.128, L1 bypass; 8-byte when VP % 4 != 0), D-1 rows ahead
+//    of the row being computed; every lane copies exactly the columns it later reads, so the ring
+//    needs no warp synchronisation at all.  (MODE 1 / 2: bulk / 2-D tensor TMA instead --
+//    measured slower, kept selectable.)
+//  * Table edges: out-of-table cells are never forced; column 0's UL and column W-1's UR take
+//    f's boundary value (the edge warps would otherwise pace everyone through the exchange).
 //  * The last band writes last_row and the row minimum (score).
+//  * prevrow_gh_kernel (below): lane-ghost variant, measured slower, kept selectable.
 #include <cstdint>
 #include <climits>
 #include "cellfn.cuh"
