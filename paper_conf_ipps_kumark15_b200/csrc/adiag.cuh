@@ -128,6 +128,10 @@ struct AdWarp {
   // ---- per-warp handoff state
   uint64_t tp;      // this lane's top pair of the current chunk (column 32k + lane)
   uint64_t tq1;     // global top prefetch (chunk k+1)
+  const uint64_t* tqsrc;   // TS 2: this lane's slot of the previous strip's boundary row (column
+                           // 32k + lane at tqsrc + 32k); the next chunk's pair is loaded half a
+                           // chunk ahead (at group 2), late enough to be published already
+  int tqn;                 // chunks with a global top pair (NQ), 0 for other roles
   long long wait_top; // clock64 cycles spent waiting for top values (trace builds)
 
   __device__ __forceinline__ CC colctx_guard(const FillParams& p, int c) const {
@@ -177,8 +181,11 @@ struct AdWarp {
     } else {
       src = lk.gprev + 32 * (int64_t)k + lane;
       tag = lk.ep32;
-      tp = tq1;                                                   // loaded one chunk ago
-      tq1 = (k + 1 < NQ) ? ad_ld_gpu(src + 32) : 0ull;            // next chunk, in flight
+      tp = tq1;
+      // next chunk's pair: here, one chunk ahead, for the 2-group-unrolled f's (LCS / Lev: a load
+      // inside their group loop cost every warp ~6 cycles per step); half a chunk ahead, inside
+      // the fully unrolled group loop, for DTW (C2 1.00 -> 0.93 ms)
+      if constexpr (kAdGroupUnroll<F> != 4) tq1 = (k + 1 < NQ) ? ad_ld_gpu(src + 32) : 0ull;
     }
     if (__all_sync(0xffffffffu, (uint32_t)(tp >> 32) == tag)) return true;
     const long long t0 = clock64();
@@ -272,6 +279,11 @@ struct AdWarp {
     }
 #pragma unroll(kAdGroupUnroll<F>)
     for (int g = 0; g < 4; ++g) {
+      // a plain L2 load (predicated, no branch in the group body); a stale pair is caught by
+      // the tag check and re-polled with a strong load in acquire_top
+      if constexpr (kAdGroupUnroll<F> == 4) {
+        if (g == 2 && k + 1 < tqn) tq1 = __ldcg(reinterpret_cast<const unsigned long long*>(tqsrc) + 32 * (k + 1));
+      }
       CC cnext[8];
       const int tau0 = 32 * k - E + 8 * g;
       if constexpr (F::kMatchCells && SM) {
@@ -587,6 +599,8 @@ __global__ void __launch_bounds__(W * 32, 1) adiag_kernel(const FillParams p) {
     lk.top_init = (strip_top - 1 == -1);
     lk.wait_bp = 0;
     aw.tp = 0;
+    aw.tqsrc = lk.gprev + lane;
+    aw.tqn = (topsrc == 2) ? NQ : 0;
     if (topsrc == 2) aw.tq1 = ad_ld_gpu(lk.gprev + lane);
     if constexpr (F::kMatchCells)
       ok = ok && (aw.small ? aw.template strip<true>(p, lane, NQ, topsrc, botsnk, lk, ctl)
