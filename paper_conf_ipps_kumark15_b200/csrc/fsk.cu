@@ -28,6 +28,9 @@
 
 namespace lddp {
 
+#ifndef LDDP_FSK_PG
+#define LDDP_FSK_PG 2   // group of a chunk at which the next chunk's strip-boundary pair is loaded
+#endif
 namespace {
 constexpr int kFsIn = 8;     // input chunks (16 B) per lane ring
 constexpr int kFsAhead = 6;  // chunks issued ahead of the lane's current chunk
@@ -177,8 +180,7 @@ __global__ void __launch_bounds__(W * 32, 1) fsk_kernel(const FillParams p) {
           } else {
             src = gprev + 32 * (int64_t)k + lane;
             tag = ep32;
-            tp = tq1;
-            tq1 = (k + 1 < NQ) ? ad_ld_gpu(src + 32) : 0ull;
+            tp = tq1;   // loaded half a chunk ago (group 2 of the previous chunk)
           }
           if (!__all_sync(0xffffffffu, (uint32_t)(tp >> 32) == tag)) {
             Backoff bo;
@@ -211,6 +213,10 @@ __global__ void __launch_bounds__(W * 32, 1) fsk_kernel(const FillParams p) {
       // ---- 32 steps: tau = 32k - OFS + su (fully unrolled: the period test below is static)
 #pragma unroll
       for (int g = 0; g < 4; ++g) {
+        // the next chunk's strip-boundary pair, half a chunk ahead: late enough that the producer
+        // has usually published it (a stale pair is caught by the tag check and re-polled)
+        if (g == LDDP_FSK_PG && topsrc == 2 && k + 1 < NQ)
+          tq1 = __ldcg(reinterpret_cast<const unsigned long long*>(gprev) + 32 * (k + 1) + lane);
         float bv[8];
         float inn[R][8], injn[8];
         if (g < 3) {
