@@ -511,6 +511,16 @@ lddp_status lddp_plan(const lddp_desc* desc, lddp_plan_t* out) {
       int Eq = env_int("LDDP_AD_E", 0);
       int Wq = d.tile_warps > 0 ? d.tile_warps : env_int("LDDP_AD_W", 0);
       int Sq = env_int("LDDP_AD_S", -1);
+      // DTW: one warp per strip (every handoff through the global boundary rows, prefetched half
+      // a chunk ahead) measured best on B200 (C2 0.93 -> 0.85 ms against 4-warp CTAs)
+      if (Wq <= 0 && d.func == LDDP_F_DTW) Wq = 1;
+      // LCS / Levenshtein: one warp per strip too when the strips of 192 rows fit one wave of
+      // CTAs (small tables, C1 0.084 -> 0.080 ms); 4-warp CTAs with shared rings otherwise
+      // (C5: 521 one-warp strips measured 8.2 ms against 6.6)
+      if (Wq <= 0 && d.func != LDDP_F_DTW && (d.rows + 191) / 192 <= pl->sms) {
+        for (const auto& g : kAdGeoms)
+          if (g.func == d.func && g.W == 1) { Wq = 1; break; }
+      }
       double best = 1e300;
       pl->R = 0;
       for (const auto& g : kAdGeoms) {
