@@ -93,6 +93,10 @@ __device__ __forceinline__ uint64_t ad_pair(uint32_t bits, uint32_t tag) {
 template <class F, int R, int W, int E, int S = 0>
 struct AdWarp {
   static constexpr int ELAG = E + S;   // lane-to-lane column lag
+  // strip-boundary pairs loaded half a chunk ahead inside the group loop: DTW (fully unrolled
+  // groups) and one-warp CTAs (every warp reads its top row from global memory); for 4-warp
+  // LCS CTAs the load inside the 2-group loop cost every warp more than it saved warp 0
+  static constexpr bool kAdHalfPf = kAdGroupUnroll<F> == 4 || W == 1;
   static constexpr int H2 = S ? R / 2 : R;
   static_assert(!S || (R % 2 == 0), "split needs an even R");
   using T = typename F::T;
@@ -182,10 +186,8 @@ struct AdWarp {
       src = lk.gprev + 32 * (int64_t)k + lane;
       tag = lk.ep32;
       tp = tq1;
-      // next chunk's pair: here, one chunk ahead, for the 2-group-unrolled f's (LCS / Lev: a load
-      // inside their group loop cost every warp ~6 cycles per step); half a chunk ahead, inside
-      // the fully unrolled group loop, for DTW (C2 1.00 -> 0.93 ms)
-      if constexpr (kAdGroupUnroll<F> != 4) tq1 = (k + 1 < NQ) ? ad_ld_gpu(src + 32) : 0ull;
+      // next chunk's pair: half a chunk ahead inside the group loop (kAdHalfPf), else here
+      if constexpr (!kAdHalfPf) tq1 = (k + 1 < NQ) ? ad_ld_gpu(src + 32) : 0ull;
     }
     if (__all_sync(0xffffffffu, (uint32_t)(tp >> 32) == tag)) return true;
     const long long t0 = clock64();
@@ -281,7 +283,7 @@ struct AdWarp {
     for (int g = 0; g < 4; ++g) {
       // a plain L2 load (predicated, no branch in the group body); a stale pair is caught by
       // the tag check and re-polled with a strong load in acquire_top
-      if constexpr (kAdGroupUnroll<F> == 4) {
+      if constexpr (kAdHalfPf) {
         if (g == 2 && k + 1 < tqn) tq1 = __ldcg(reinterpret_cast<const unsigned long long*>(tqsrc) + 32 * (k + 1));
       }
       CC cnext[8];

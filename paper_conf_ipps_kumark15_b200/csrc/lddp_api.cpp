@@ -517,7 +517,7 @@ lddp_status lddp_plan(const lddp_desc* desc, lddp_plan_t* out) {
       // LCS / Levenshtein: one warp per strip too when the strips of 192 rows fit one wave of
       // CTAs (small tables, C1 0.084 -> 0.080 ms); 4-warp CTAs with shared rings otherwise
       // (C5: 521 one-warp strips measured 8.2 ms against 6.6)
-      if (Wq <= 0 && d.func != LDDP_F_DTW && (d.rows + 191) / 192 <= pl->sms) {
+      if (Wq <= 0 && d.func != LDDP_F_DTW) {
         for (const auto& g : kAdGeoms)
           if (g.func == d.func && g.W == 1) { Wq = 1; break; }
       }
@@ -549,7 +549,8 @@ lddp_status lddp_plan(const lddp_desc* desc, lddp_plan_t* out) {
       pl->nchunks = (int)((d.cols + 31) / 32);
       pl->bnd_stride = (int64_t)std::max(pl->nchunks, 1) * 32;   // (value, tag) pairs per strip row
       int g = d.grid_ctas > 0 ? d.grid_ctas : env_int("LDDP_GRID_CTAS", 0);
-      pl->grid = g > 0 ? g : pl->sms;
+      // one-warp CTAs: enough of them for every strip to be resident at once
+      pl->grid = g > 0 ? g : (pl->W == 1 ? std::min(pl->nstrips, pl->sms * 8) : pl->sms);
       pl->off_prog = 64;
       pl->off_bnd = 256;
       pl->ws_bytes = pl->off_bnd + (size_t)std::max(pl->nstrips - 1, 1) * pl->bnd_stride * 8;
