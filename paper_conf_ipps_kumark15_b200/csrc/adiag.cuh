@@ -36,6 +36,16 @@ namespace lddp {
 
 // 8-step groups per loop iteration (measured on B200: LCS / Levenshtein 2, DTW 4 -- C5 8.36 ->
 // 7.86 ms, C2 1.13 -> 1.00 ms against 1; LDDP_AD_GUNROLL overrides for experiments)
+// group of a chunk at which the next chunk's strip-boundary pairs are loaded (kAdHalfPf); measured
+// on B200: LCS C5 6.27 / 6.12 / 5.80 ms at group 2 / 1 / 0 -- an early load hides the L2 latency
+// better than a stale pair costs
+#ifndef LDDP_AD_PG_MATCH
+#define LDDP_AD_PG_MATCH 0
+#endif
+#ifndef LDDP_AD_PG_OTHER
+#define LDDP_AD_PG_OTHER 2
+#endif
+template <class F> constexpr int kAdPfGroup = F::kMatchCells ? LDDP_AD_PG_MATCH : LDDP_AD_PG_OTHER;
 #ifdef LDDP_AD_GUNROLL
 template <class F> constexpr int kAdGroupUnroll = LDDP_AD_GUNROLL;
 #else
@@ -284,7 +294,7 @@ struct AdWarp {
       // a plain L2 load (predicated, no branch in the group body); a stale pair is caught by
       // the tag check and re-polled with a strong load in acquire_top
       if constexpr (kAdHalfPf) {
-        if (g == 2 && k + 1 < tqn) tq1 = __ldcg(reinterpret_cast<const unsigned long long*>(tqsrc) + 32 * (k + 1));
+        if (g == kAdPfGroup<F> && k + 1 < tqn) tq1 = __ldcg(reinterpret_cast<const unsigned long long*>(tqsrc) + 32 * (k + 1));
       }
       CC cnext[8];
       const int tau0 = 32 * k - E + 8 * g;
