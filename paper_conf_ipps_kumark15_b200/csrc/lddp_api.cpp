@@ -387,6 +387,17 @@ lddp_status launch(lddp_plan_t pl, const FillParams& p, cudaStream_t s) {
   } else if (pl->kind == 3) {
     int grid = std::min(pl->grid, p.nstrips);
     e = pl->ad_launch(p, grid, s);
+  } else if (pl->kind == 4 && (reinterpret_cast<uintptr_t>(p.b) & 3) == 0) {
+    int grid = std::min(pl->grid, p.nstrips);
+    e = lddp::launch_lcs16(p, pl->R, pl->E, grid, s);
+  } else if (pl->kind == 4) {
+    // b not 4-byte aligned (lcs16 copies it in 4-byte granules): the 32-bit adiag kernel
+    FillParams q = p;
+    q.nstrips = (int)((pl->desc.rows + 191) / 192);
+    q.row0 = pl->desc.rows - (int64_t)q.nstrips * 192;
+    q.strip_rows = 192;
+    q.bnd_stride = (int64_t)std::max((q.cols + 31) / 32, 1) * 32;
+    e = lddp::ad_lcs_r6e2w1(q, std::min(q.nstrips, pl->sms * 8), s);
   } else if (pl->kind == 1 && pl->cb_variant >= 0 && (p.grid_pitch % 4 == 0) &&
              ((reinterpret_cast<uintptr_t>(p.grid) & 15) == 0)) {
     FillParams q = p;
@@ -504,7 +515,37 @@ lddp_status lddp_plan(const lddp_desc* desc, lddp_plan_t* out) {
 
     const char* kern_env = getenv("LDDP_KERNEL");
     const bool force_wf = kern_env != nullptr && strcmp(kern_env, "wavefront") == 0;
-    if (d.category == LDDP_CAT_ANTI_DIAGONAL && seq_func(d.func) && !table && !force_wf) {
+    const bool force_ad = kern_env != nullptr && strcmp(kern_env, "adiag") == 0;
+    if (d.category == LDDP_CAT_ANTI_DIAGONAL && d.func == LDDP_F_LCS && !table && !force_wf && !force_ad) {
+      // packed 16x2 LCS kernel (lcs16.cu): P row pairs per lane, lane lag E
+      pl->kind = 4;
+      pl->R = d.tile_rows > 0 ? (d.tile_rows + 1) / 2 : env_int("LDDP_L16_P", 3);
+      pl->E = env_int("LDDP_L16_E", 3);
+      pl->W = 1;
+      pl->SIG = 0;
+      if (!lddp::lcs16_compiled(pl->R, pl->E)) {
+        const int P = pl->R, E = pl->E;
+        delete pl;
+        return fail(LDDP_ERR_UNSUPPORTED, "lcs16 P=%d E=%d not compiled", P, E);
+      }
+      pl->variant = -1;
+      pl->occupancy = 1;
+      pl->strip_rows = (int64_t)64 * pl->R;
+      pl->nstrips = (int)((d.rows + pl->strip_rows - 1) / pl->strip_rows);
+      pl->row0 = d.rows - (int64_t)pl->nstrips * pl->strip_rows;
+      pl->nchunks = (int)((d.cols + 31) / 32);
+      pl->bnd_stride = (int64_t)std::max(pl->nchunks, 1) * 32;
+      int g = d.grid_ctas > 0 ? d.grid_ctas : env_int("LDDP_GRID_CTAS", 0);
+      // grid = strip workers (warps), packed 4 per CTA: one warp per SM sub-partition
+      pl->grid = g > 0 ? g : std::min(pl->nstrips, pl->sms * 4);
+      pl->off_prog = 64;
+      pl->off_bnd = 256;
+      // boundary rows for lcs16's strips, or for the 192-row strips of the adiag fallback (b not
+      // 4-byte aligned), whichever is more
+      const int64_t fb_strips = (d.rows + 191) / 192;
+      pl->ws_bytes = pl->off_bnd + (size_t)std::max<int64_t>(std::max(pl->nstrips, (int)fb_strips) - 1, 1) *
+                                       pl->bnd_stride * 8;
+    } else if (d.category == LDDP_CAT_ANTI_DIAGONAL && seq_func(d.func) && !table && !force_wf) {
       // lane-systolic anti-diagonal kernel (adiag.cuh)
       pl->kind = 3;
       int Rq = d.tile_rows > 0 ? d.tile_rows : env_int("LDDP_AD_R", 0);
@@ -677,7 +718,7 @@ lddp_status lddp_plan_workspace_size(lddp_plan_t pl, size_t* bytes) {
 
 lddp_status lddp_plan_describe(lddp_plan_t pl, char* buf, size_t len) {
   if (pl == nullptr || buf == nullptr || len == 0) return fail(LDDP_ERR_INVALID_ARG, "NULL argument");
-  static const char* kinds[] = {"wavefront", "prevrow", "invl", "adiag"};
+  static const char* kinds[] = {"wavefront", "prevrow", "invl", "adiag", "lcs16"};
   const bool cb = pl->kind == 1 && pl->cb_variant >= 0;
   if (pl->kind == 0 && pl->fsk) {
     snprintf(buf, len,
@@ -696,7 +737,7 @@ lddp_status lddp_plan_describe(lddp_plan_t pl, char* buf, size_t len) {
            "\"strips\": %d, \"chunks\": %d, \"blocks\": %d, \"bands\": %d, \"workspace_bytes\": %zu}",
            cb ? "prevrow_cb" : kinds[pl->kind], cb ? pl->cb_variant : pl->variant, pl->R, pl->SIG, pl->E,
            cb ? pl->cb_nw
-              : (pl->kind == 0 ? kWfWarps + 2 : (pl->kind == 1 ? kPrevThreads / 32 : (pl->kind == 3 ? pl->W : kInvlThreads / 32))),
+              : (pl->kind == 0 ? kWfWarps + 2 : (pl->kind == 1 ? kPrevThreads / 32 : (pl->kind >= 3 ? pl->W : kInvlThreads / 32))),
            cb ? (pl->cb_nblocks + pl->cb_nw - 1) / pl->cb_nw : pl->grid,
            pl->sms, cb ? 1 : pl->occupancy, (long long)pl->strip_rows, pl->nstrips, pl->nchunks,
            cb ? pl->cb_nblocks : pl->nblocks, pl->nbands, pl->ws_bytes);
@@ -819,7 +860,7 @@ lddp_status lddp_status_check(lddp_plan_t pl, void* ws, void* stream) {
 lddp_status lddp_comm_create(lddp_plan_t pl, int32_t nranks, int32_t rank, lddp_comm_t* out) {
   if (pl == nullptr || out == nullptr) return fail(LDDP_ERR_INVALID_ARG, "NULL argument");
   if (nranks < 1 || rank < 0 || rank >= nranks) return fail(LDDP_ERR_INVALID_ARG, "bad rank %d / %d", rank, nranks);
-  if ((pl->kind != 0 && pl->kind != 3) || pl->desc.category != LDDP_CAT_ANTI_DIAGONAL)
+  if ((pl->kind != 0 && pl->kind != 3 && pl->kind != 4) || pl->desc.category != LDDP_CAT_ANTI_DIAGONAL)
     return fail(LDDP_ERR_UNSUPPORTED, "multi-GPU column strips: anti-diagonal category only in this build");
   if (pl->desc.cols < nranks) return fail(LDDP_ERR_SHAPE, "cols < nranks");
   DeviceGuard dg(pl->desc.device);
@@ -944,7 +985,7 @@ lddp_status lddp_fill_multi(lddp_plan_t pl, const lddp_inputs* in, const lddp_ou
     p.cols = (int32_t)(c1 - c0);
     p.col0 = (int32_t)c0;
     p.cols_total = (int32_t)n;
-    if (pl->kind == 3) {
+    if (pl->kind == 3 || pl->kind == 4) {
       p.nchunks = (int)((p.cols + 31) / 32);
       p.bnd_stride = (int64_t)std::max(p.nchunks, 1) * 32;
     } else {

@@ -53,6 +53,7 @@ struct FillParams {
   int32_t one;              // always 1 (a run-time constant the compiler cannot fold)
   int32_t spin_polls;       // polls before a waiting warp starts to back off (env LDDP_SPIN)
   int32_t debug;            // env LDDP_DEBUG bits (development): 1 = adiag warps without handoffs
+  int32_t workers;          // lcs16: persistent strip workers (warps); extra warps of the last CTA idle
 };
 
 // Launch entry points (one per category family).  Return cudaError_t of the launch.
@@ -69,6 +70,9 @@ cudaError_t launch_fsk(const FillParams& p, int W, int E, int R, int grid, cudaS
 cudaError_t launch_traceback(int func, const void* a, const void* b, const void* table, int64_t pitch, int64_t m,
                              int64_t n, int32_t* pi, int32_t* pj, int64_t* len, cudaStream_t s);
 cudaError_t launch_invl(int func, const FillParams& p, int grid, cudaStream_t stream);
+// Packed 16x2 LCS kernel (lcs16.cu): P row pairs per lane (strips of 64P rows), lane lag E.
+cudaError_t launch_lcs16(const FillParams& p, int P, int E, int grid, cudaStream_t stream);
+bool lcs16_compiled(int P, int E);
 
 // Per-kernel occupancy query (blocks per SM) for the chosen configuration.
 int wavefront_blocks_per_sm(int func, int category, int rows_per_lane, int warps);

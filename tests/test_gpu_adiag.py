@@ -43,7 +43,8 @@ def _check(func, got, ref):
 
 
 def _run(func, R, E, W, a, b, S=0, **kw):
-    old = {k: os.environ.get(k) for k in ("LDDP_AD_E", "LDDP_AD_W", "LDDP_AD_S")}
+    old = {k: os.environ.get(k) for k in ("LDDP_AD_E", "LDDP_AD_W", "LDDP_AD_S", "LDDP_KERNEL")}
+    os.environ["LDDP_KERNEL"] = "adiag"   # LCS defaults to lcs16.cu (test_gpu_lcs16.py)
     os.environ["LDDP_AD_E"] = str(E)
     os.environ["LDDP_AD_W"] = str(W)
     os.environ["LDDP_AD_S"] = str(S)
@@ -95,7 +96,7 @@ def test_adiag_large(func):
     m, n = 6001, 5003
     a, b = _inputs(func, 77, m, n)
     got = run_gpu(func, "anti_diagonal", a=a, b=b, outputs=("score", "last_row", "last_col"), reps=2)
-    assert '"adiag"' in got["plan"]
+    assert ('"lcs16"' if func == "lcs" else '"adiag"') in got["plan"]
     _check(func, got, _ref(func, a, b))
 
 
