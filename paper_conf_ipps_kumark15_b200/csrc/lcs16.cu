@@ -67,11 +67,27 @@ __device__ __forceinline__ void cp_async_cg16(void* dst, const void* src) {
 }
 __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
 
+// opaque register copies: ptxas cannot rematerialise them from the constant bank inside the loop
+__device__ __forceinline__ int opq(int x) {
+  asm volatile("mov.b32 %0, %0;" : "+r"(x));
+  return x;
+}
+template <class T>
+__device__ __forceinline__ T* opqp(T* x) {
+  asm volatile("mov.b64 %0, %0;" : "+l"(x));
+  return x;
+}
+
 constexpr int kRing = 256;    // column ring entries (index = column & 255) + 8 mirrored
 constexpr int kChr = 1024;    // byte ring of b (index = global byte offset & 1023)
 constexpr int kPfGroup = 2;   // group of chunk k at which chunk k+1's top pairs are copied
 
 }  // namespace l16
+
+// compiled (P row pairs per lane, E lane lag) geometries
+#define LDDP_L16_GEOMS \
+  LDDP_L16_GEOM(3, 3) LDDP_L16_GEOM(3, 2) LDDP_L16_GEOM(4, 3) LDDP_L16_GEOM(4, 2) LDDP_L16_GEOM(2, 3) \
+  LDDP_L16_GEOM(3, 4)
 
 template <int P, int E>
 struct L16Warp {
@@ -98,11 +114,10 @@ struct L16Warp {
   uint32_t sq[8];       // ring selectors of the current 8-step group (loaded one group ahead)
   long long wait_top;
   uint64_t t_first;     // trace builds: globaltimer after chunk 0's top row was acquired
-  long long cyc_pre, cyc_body;   // trace builds: cycles before / in the chunk bodies
 
   // character of local column c, -1 outside [0, n) (matches nothing)
-  __device__ __forceinline__ int32_t chr_at(const FillParams& p, int c) const {
-    return ((unsigned)c < (unsigned)p.cols) ? (int32_t)chr[(p.col0 + c) & (l16::kChr - 1)] : -1;
+  __device__ __forceinline__ int32_t chr_at(int cols, int col0, int c) const {
+    return ((unsigned)c < (unsigned)cols) ? (int32_t)chr[(col0 + c) & (l16::kChr - 1)] : -1;
   }
   template <bool SM>
   __device__ __forceinline__ uint32_t ring_entry(int32_t ca, int32_t cb) const {
@@ -130,12 +145,18 @@ struct L16Warp {
     return 0;   // table row 0 (i = -1) and the virtual rows above it: LCS boundary 0
   }
 
+  // Per-strip loop state in registers (opaque copies of FillParams fields and per-lane pointers,
+  // advanced by one chunk per iteration).
   struct Links {
-    const uint64_t* gprev;   // strip s-1's boundary row
-    uint64_t* gmine;         // strip s's boundary row
+    const uint64_t* gprev;   // strip s-1's boundary row (base)
+    uint64_t* gmine;         // strip s's boundary row (base)
     int32_t* stg;            // bottom staging row (packed, relative to the chunk's base)
     int32_t* tstg;           // top staging row (relative lo halves)
     uint32_t ep32;
+    int cols, col0, btot, wlim;
+    const uint64_t* pf;      // prefetch source of chunk k+1: gprev + 32(k+1) + 2 lane
+    uint64_t* pub;           // publish target of chunk k-1-ELAG: gmine + 32(k-1-ELAG) + lane
+    int32_t* lrow;           // last_row + 32(k-1-ELAG) + lane (BS 3)
   };
 
   // Top pairs of chunk k (columns 32k + lane), validated before the chunk's steps run.
@@ -157,25 +178,24 @@ struct L16Warp {
     wait_top += clock64() - t0;
     return true;
   }
+  // chunk k+1's top pairs -> pbuf (lanes 0..15, 16 bytes each)
   template <int TS>
-  __device__ __forceinline__ void prefetch_top(int lane, int k, int NQ, const Links& lk) {
-    if (TS == 2 && k < NQ && lane < 16) l16::cp_async_cg16(pbuf + 2 * lane, lk.gprev + 32 * k + 2 * lane);
+  __device__ __forceinline__ void prefetch_top(int lane, int k1, int NQ, const Links& lk) {
+    if (TS == 2 && k1 < NQ && lane < 16) l16::cp_async_cg16(pbuf + 2 * lane, lk.pf);
     cp_async_commit();
   }
 
   // Bottom chunk j (columns 32j + lane): staged by lane 31 during the chunk that produced it.
   // BS 2: boundary row of this strip (pairs); 3: the last_row output; 0: nothing.
   template <int BS>
-  __device__ __forceinline__ void publish_bottom(const FillParams& p, int lane, int j, int NQ, const Links& lk) {
+  __device__ __forceinline__ void publish_bottom(int lane, int j, int NQ, const Links& lk) {
     if (BS == 0 || j < 0 || j >= NQ) return;
     __syncwarp();
     const int32_t v = (int32_t)((uint32_t)lk.stg[lane] >> 16) + base;
     if (BS == 2) {
-      uint64_t* d = lk.gmine + 32 * j + lane;
-      asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(d), "l"(ad_pair((uint32_t)v, lk.ep32)) : "memory");
+      asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(lk.pub), "l"(ad_pair((uint32_t)v, lk.ep32)) : "memory");
     } else {
-      const int c = 32 * j + lane;
-      if (c < p.cols) static_cast<int32_t*>(p.last_row)[c] = v;
+      if (32 * j + lane < lk.cols) *lk.lrow = v;
     }
   }
 
@@ -196,17 +216,16 @@ struct L16Warp {
 
   // One chunk = 32 steps tau = 32k - E + su in 4 groups of 8.
   template <bool SM, int TS>
-  __device__ __forceinline__ void chunk(const FillParams& p, const int lane, const int k, const int NQ,
-                                        const Links& lk, const int w0, const int wlim) {
+  __device__ __forceinline__ void chunk(const int lane, const int k, const int NQ, const Links& lk, const int w0) {
     const int lane_off = lane * E;
     {   // column ring: the entry of column 32(k+1) + lane
       const int c = 32 * (k + 1) + lane;
       const int slot = c & (l16::kRing - 1);
-      const uint32_t v = ring_entry<SM>(chr_at(p, c), chr_at(p, c - 32 * E));
+      const uint32_t v = ring_entry<SM>(chr_at(lk.cols, lk.col0, c), chr_at(lk.cols, lk.col0, c - 32 * E));
       ring[slot] = v;
       if (slot < 8) ring[slot + l16::kRing] = v;
     }
-    copy_chars(lane, w0, wlim, p.cols_total);   // columns 32(k+2) ..
+    copy_chars(lane, w0, lk.wlim, lk.btot);   // columns 32(k+2) ..
     // chunk k's top row (relative) -> shared memory; lane 31 injects it one group ahead.  Past
     // the last chunk any value <= the rows' own keeps them constant: 0 (relative values are >= 0)
     lk.tstg[lane] = k < NQ ? max((int32_t)(uint32_t)tp - base, 0) : 0;
@@ -287,15 +306,20 @@ struct L16Warp {
   }
 
   template <bool SM, int TS, int BS>
-  __device__ __forceinline__ bool strip(const FillParams& p, int lane, int NQ, const Links& lk, Control* ctl) {
+  __device__ __forceinline__ bool strip(const FillParams& p, int lane, int NQ, Links lk, Control* ctl) {
     const int K = NQ + ELAG;
-    const bool trace = p.trace != nullptr;
-    const int wlim = (p.cols_total + 3) >> 2;
-    int w0 = ((p.col0 + 64) >> 2);   // granule of column 32(k+2) at k = 0 (8 granules per chunk)
-    for (int k = 0; k < K; ++k, w0 += 8) {
-      long long c0 = 0;
-      if (trace) c0 = clock64();
-      publish_bottom<BS>(p, lane, k - 1 - ELAG, NQ, lk);   // staged during chunk k-1 (its base)
+    const bool trace = l16::opq(p.trace != nullptr ? 1 : 0) != 0;
+    lk.cols = l16::opq(p.cols);
+    lk.col0 = l16::opq(p.col0);
+    lk.btot = l16::opq(p.cols_total);
+    lk.wlim = (lk.btot + 3) >> 2;
+    lk.ep32 = (uint32_t)l16::opq((int)lk.ep32);
+    lk.pf = l16::opqp(lk.gprev + 32 + 2 * lane);
+    lk.pub = l16::opqp(lk.gmine + lane - 32 * (1 + ELAG));
+    lk.lrow = l16::opqp(static_cast<int32_t*>(p.last_row) + lane - 32 * (1 + ELAG));
+    int w0 = ((lk.col0 + 64) >> 2);   // granule of column 32(k+2) at k = 0 (8 granules per chunk)
+    for (int k = 0; k < K; ++k) {
+      publish_bottom<BS>(lane, k - 1 - ELAG, NQ, lk);   // staged during chunk k-1 (its base)
       // every 8 chunks (a chunk adds at most 32 to any value: 16 bits keep > 60000 of headroom)
       if ((k & 7) == 0 && k > 0) rebase();
       // chunk k-1's copies (characters of columns 32(k+1).., chunk k's top pairs) have landed
@@ -303,17 +327,14 @@ struct L16Warp {
       __syncwarp();
       if (!acquire_top<TS>(p, lane, k, NQ, lk, ctl)) return false;
       if (trace && k == 0) t_first = globaltimer_ns();
-      long long c1 = 0;
-      if (trace) c1 = clock64();
-      chunk<SM, TS>(p, lane, k, NQ, lk, w0, wlim);
-      if (trace) {
-        const long long c2 = clock64();
-        cyc_pre += c1 - c0;
-        cyc_body += c2 - c1;
-      }
+      chunk<SM, TS>(lane, k, NQ, lk, w0);
+      w0 += 8;
+      lk.pf += 32;
+      lk.pub += 32;
+      lk.lrow += 32;
     }
     l16::cp_async_wait_all();
-    publish_bottom<BS>(p, lane, K - 1 - ELAG, NQ, lk);
+    publish_bottom<BS>(lane, K - 1 - ELAG, NQ, lk);
     return true;
   }
   template <bool SM>
@@ -450,7 +471,7 @@ __global__ void __launch_bounds__(32 * WPC, 1) lcs16_kernel(const FillParams p) 
     __syncwarp();
     for (int q = -E - 1; q <= 0; ++q) {
       const int c = 32 * q + lane;
-      const int32_t ca = lw.chr_at(p, c), cb = lw.chr_at(p, c - 32 * E);
+      const int32_t ca = lw.chr_at(n, p.col0, c), cb = lw.chr_at(n, p.col0, c - 32 * E);
       const uint32_t v = small ? lw.template ring_entry<true>(ca, cb) : lw.template ring_entry<false>(ca, cb);
       const int slot = c & (l16::kRing - 1);
       ring[slot] = v;
@@ -466,8 +487,6 @@ __global__ void __launch_bounds__(32 * WPC, 1) lcs16_kernel(const FillParams p) 
     const long long ck0 = clock64();
     lw.wait_top = 0;
     lw.t_first = 0;
-    lw.cyc_pre = 0;
-    lw.cyc_body = 0;
     typename LW::Links lk;
     lk.gprev = static_cast<const uint64_t*>(p.bnd) + (int64_t)(s - 1) * p.bnd_stride;
     lk.gmine = static_cast<uint64_t*>(p.bnd) + (int64_t)s * p.bnd_stride;
@@ -476,7 +495,10 @@ __global__ void __launch_bounds__(32 * WPC, 1) lcs16_kernel(const FillParams p) 
     lk.ep32 = (uint32_t)p.epoch;
     lw.tp = 0;
     lw.bsrc = static_cast<const uint8_t*>(p.b);
-    if (TS == 2) lw.template prefetch_top<2>(lane, 0, NQ, lk);   // chunk 0's top pairs
+    if (TS == 2) {   // chunk 0's top pairs
+      lk.pf = lk.gprev + 2 * lane;
+      lw.template prefetch_top<2>(lane, 0, NQ, lk);
+    }
     ok = ok && (small ? lw.template strip_roles<true>(p, lane, NQ, TS, BS, lk, ctl)
                       : lw.template strip_roles<false>(p, lane, NQ, TS, BS, lk, ctl));
     if (p.trace != nullptr && lane == 0) {
@@ -490,8 +512,8 @@ __global__ void __launch_bounds__(32 * WPC, 1) lcs16_kernel(const FillParams p) 
       asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
       asm volatile("mov.u32 %0, %%warpid;" : "=r"(warpid));
       tr[5] = ((uint64_t)smid << 32) | warpid;
-      tr[6] = (uint64_t)lw.cyc_pre;
-      tr[7] = (uint64_t)lw.cyc_body;
+      tr[6] = 0;
+      tr[7] = 0;
     }
     // right column = the final registers (rows keep their column n-1 value past the end)
     if (ok) {
@@ -539,14 +561,18 @@ cudaError_t lcs16_launch(const FillParams& p, int warps, cudaStream_t s) {
 // Compiled geometries (P pairs = 2P rows per lane, E steps of lane lag); `warps` persistent
 // strip workers (rounded up to whole 4-warp CTAs).  b must be 4-byte aligned (cp.async granules).
 cudaError_t launch_lcs16(const FillParams& p, int P, int E, int warps, cudaStream_t s) {
-  if (P == 3 && E == 3) return lcs16_launch<3, 3>(p, warps, s);
-  if (P == 3 && E == 4) return lcs16_launch<3, 4>(p, warps, s);
-  if (P == 4 && E == 3) return lcs16_launch<4, 3>(p, warps, s);
-  if (P == 2 && E == 3) return lcs16_launch<2, 3>(p, warps, s);
+#define LDDP_L16_GEOM(PP, EE) \
+  if (P == PP && E == EE) return lcs16_launch<PP, EE>(p, warps, s);
+  LDDP_L16_GEOMS
+#undef LDDP_L16_GEOM
   return cudaErrorInvalidValue;
 }
 bool lcs16_compiled(int P, int E) {
-  return (P == 3 && (E == 3 || E == 4)) || (P == 4 && E == 3) || (P == 2 && E == 3);
+#define LDDP_L16_GEOM(PP, EE) \
+  if (P == PP && E == EE) return true;
+  LDDP_L16_GEOMS
+#undef LDDP_L16_GEOM
+  return false;
 }
 
 }  // namespace lddp
