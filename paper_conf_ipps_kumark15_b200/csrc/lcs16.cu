@@ -81,19 +81,20 @@ __device__ __forceinline__ T* opqp(T* x) {
 constexpr int kRing = 256;    // column ring entries (index = column & 255) + 8 mirrored
 constexpr int kChr = 1024;    // byte ring of b (index = global byte offset & 1023)
 constexpr int kPfGroup = 2;   // group of chunk k at which chunk k+1's top pairs are copied
+constexpr int kDynPerWarp = 257 * 32 * 2;   // table path: 257 characters x 32 lanes x u16
 
 }  // namespace l16
 
 // compiled (P row pairs per lane, E lane lag) geometries
 #define LDDP_L16_GEOMS \
   LDDP_L16_GEOM(3, 3) LDDP_L16_GEOM(3, 2) LDDP_L16_GEOM(4, 3) LDDP_L16_GEOM(4, 2) LDDP_L16_GEOM(2, 3) \
-  LDDP_L16_GEOM(3, 4)
+  LDDP_L16_GEOM(6, 2) LDDP_L16_GEOM(6, 3) LDDP_L16_GEOM(8, 2) LDDP_L16_GEOM(8, 3)
 
 template <int P, int E>
 struct L16Warp {
   static constexpr int SH = 64 * P;     // strip rows
   static constexpr int ELAG = 2 * E;    // chunks from a top chunk to the bottom chunk it yields
-  static_assert(P >= 1 && P <= 4, "match-table entries hold 4 A rows and 4 B rows");
+  static_assert(P >= 1 && P <= 8, "match-table entries hold 8 A rows and 8 B rows");
   static_assert(32 * E + 96 <= l16::kRing, "column ring too small for the band-B lag");
 
   uint32_t h[P];        // pair p at the previous step (L of this step)
@@ -106,7 +107,7 @@ struct L16Warp {
   uint32_t* ring;       // per-warp column ring (selectors, or packed characters)
   uint8_t* chr;         // per-warp byte ring of b
   const uint8_t* ctab;  // per-warp character -> code table (small path)
-  const uint8_t* mtab;  // per-warp match table (table path): [c][lane] bits p = A rows, 4+p = B rows;
+  const uint16_t* mtab; // per-warp match table (table path): [c][lane] bits p = A rows, 8+p = B rows;
                         // row 256 stays zero (out-of-range columns)
   uint64_t* pbuf;       // per-warp next-chunk top pairs (cp.async destination)
   const uint8_t* bsrc;  // b (whole string; 4-byte aligned)
@@ -218,14 +219,6 @@ struct L16Warp {
   template <bool SM, int TS>
   __device__ __forceinline__ void chunk(const int lane, const int k, const int NQ, const Links& lk, const int w0) {
     const int lane_off = lane * E;
-    {   // column ring: the entry of column 32(k+1) + lane
-      const int c = 32 * (k + 1) + lane;
-      const int slot = c & (l16::kRing - 1);
-      const uint32_t v = ring_entry<SM>(chr_at(lk.cols, lk.col0, c), chr_at(lk.cols, lk.col0, c - 32 * E));
-      ring[slot] = v;
-      if (slot < 8) ring[slot + l16::kRing] = v;
-    }
-    copy_chars(lane, w0, lk.wlim, lk.btot);   // columns 32(k+2) ..
     // chunk k's top row (relative) -> shared memory; lane 31 injects it one group ahead.  Past
     // the last chunk any value <= the rows' own keeps them constant: 0 (relative values are >= 0)
     lk.tstg[lane] = k < NQ ? max((int32_t)(uint32_t)tp - base, 0) : 0;
@@ -239,6 +232,17 @@ struct L16Warp {
     }
 #pragma unroll
     for (int g = 0; g < 4; ++g) {
+      if (g == 1) {
+        // column ring: the entry of column 32(k+1) + lane (first read by group 3's look-ahead:
+        // placed mid-chunk so its two dependent LDS hide behind the steps), then the
+        // characters of columns 32(k+2) ..
+        const int c = 32 * (k + 1) + lane;
+        const int slot = c & (l16::kRing - 1);
+        const uint32_t v = ring_entry<SM>(chr_at(lk.cols, lk.col0, c), chr_at(lk.cols, lk.col0, c - 32 * E));
+        ring[slot] = v;
+        if (slot < 8) ring[slot + l16::kRing] = v;
+        copy_chars(lane, w0, lk.wlim, lk.btot);
+      }
       if (g == l16::kPfGroup) prefetch_top<TS>(lane, k + 1, NQ, lk);
       const int tau0 = 32 * k - E + 8 * g;
       uint32_t injn[8];
@@ -252,6 +256,7 @@ struct L16Warp {
       // the next group's selectors (group 0 of chunk k+1: its ring entries were all written by
       // the start of this chunk), loaded a group ahead so the LDS latency stays off the steps
       uint32_t sn[8];
+      if (g == 3) __syncwarp();   // group 1's ring entries are read by this look-ahead
       {
         const uint32_t* rn = ring + ((tau0 + 8 - lane_off) & (l16::kRing - 1));
 #pragma unroll
@@ -265,9 +270,9 @@ struct L16Warp {
 #pragma unroll
           for (int q = 0; q < P; ++q) mk[q] = l16::prmt(tabA[q], tabB[q], s);
         } else {
-          const uint32_t wa = mtab[(s & 0xFFFFu) * 32 + lane];
-          const uint32_t wb = mtab[(s >> 16) * 32 + lane];
-          const uint32_t comb = l16::imad(wb, 4096u, wa);   // A bits 0..3, B bits 16..19
+          const uint32_t wa = mtab[(s & 0xFFFFu) * 32 + lane] & 0xFFu;
+          const uint32_t wb = mtab[(s >> 16) * 32 + lane] >> 8;
+          const uint32_t comb = l16::imad(wb, 65536u, wa);   // A bits 0..7, B bits 16..23
 #pragma unroll
           for (int q = 0; q < P; ++q) mk[q] = (comb >> q) & 0x00010001u;
         }
@@ -364,7 +369,8 @@ __global__ void __launch_bounds__(32 * WPC, 1) lcs16_kernel(const FillParams p) 
   __shared__ __align__(16) int32_t tstg_sh[WPC][32];
   __shared__ uint8_t ctab_sh[WPC][256];
   __shared__ int one_sh[WPC];
-  extern __shared__ __align__(16) uint8_t l16_dyn[];   // match tables (table path): WPC x 257 x 32 bytes
+  // per warp: the match table of the table path (257 characters x 32 lanes x 16-bit masks)
+  extern __shared__ __align__(16) uint8_t l16_dyn[];
 
   Control* ctl = static_cast<Control*>(p.ctl);
   const int lane = threadIdx.x & 31;
@@ -373,7 +379,7 @@ __global__ void __launch_bounds__(32 * WPC, 1) lcs16_kernel(const FillParams p) 
   const int NQ = (n + 31) / 32;
   uint32_t* ring = ring_sh[wid];
   uint8_t* ctab = ctab_sh[wid];
-  uint8_t* mtab = l16_dyn + wid * 257 * 32;
+  uint16_t* mtab = reinterpret_cast<uint16_t*>(l16_dyn + wid * l16::kDynPerWarp);
   if (lane == 0) one_sh[wid] = p.one;
   __syncwarp();
 
@@ -453,13 +459,14 @@ __global__ void __launch_bounds__(32 * WPC, 1) lcs16_kernel(const FillParams p) 
         lw.tabA[q] = ka < 4 ? 1u << (8 * ka) : 0u;
         lw.tabB[q] = kb < 4 ? 1u << (8 * kb) : 0u;
       }
+
     } else {
       for (int c = 0; c < 257; ++c) mtab[c * 32 + lane] = 0;
       __syncwarp();
 #pragma unroll
       for (int q = 0; q < P; ++q) {
-        if (chA[q] >= 0) mtab[chA[q] * 32 + lane] |= (uint8_t)(1u << q);
-        if (chB[q] >= 0) mtab[chB[q] * 32 + lane] |= (uint8_t)(16u << q);
+        if (chA[q] >= 0) mtab[chA[q] * 32 + lane] |= (uint16_t)(1u << q);
+        if (chB[q] >= 0) mtab[chB[q] * 32 + lane] |= (uint16_t)(256u << q);
         lw.tabA[q] = 0;
         lw.tabB[q] = 0;
       }
@@ -480,6 +487,7 @@ __global__ void __launch_bounds__(32 * WPC, 1) lcs16_kernel(const FillParams p) 
     __syncwarp();
 #pragma unroll
     for (int u = 0; u < 8; ++u) lw.sq[u] = ring[((-E - lane * E) & (l16::kRing - 1)) + u];   // chunk 0, group 0
+
 
     const int TS = (s > 0 && !(p.debug & 2)) ? 2 : 0;   // debug 2: no strip handoff (timing only)
     const int BS = last_strip ? (p.last_row != nullptr ? 3 : 0) : 2;
@@ -551,9 +559,15 @@ __global__ void __launch_bounds__(32 * WPC, 1) lcs16_kernel(const FillParams p) 
 template <int P, int E>
 cudaError_t lcs16_launch(const FillParams& p, int warps, cudaStream_t s) {
   constexpr int WPC = 4;
-  constexpr size_t dyn = WPC * 257 * 32;
+  constexpr size_t dyn = WPC * l16::kDynPerWarp;
   FillParams q = p;
   q.workers = warps;
+  static bool attr = false;   // > 48 KB of dynamic shared memory: opt in once
+  if (!attr) {
+    cudaError_t e = cudaFuncSetAttribute(lcs16_kernel<P, E, WPC>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn);
+    if (e != cudaSuccess) return e;
+    attr = true;
+  }
   lcs16_kernel<P, E, WPC><<<(warps + WPC - 1) / WPC, 32 * WPC, dyn, s>>>(q);
   return cudaGetLastError();
 }

@@ -15,7 +15,7 @@ from paper_conf_ipps_kumark15_b200 import inputs
 
 pytestmark = pytest.mark.gpu
 
-GEOMS = [(3, 3), (3, 2), (4, 3), (4, 2), (2, 3), (3, 4)]
+GEOMS = [(3, 3), (3, 2), (4, 3), (4, 2), (2, 3), (6, 2), (6, 3), (8, 2), (8, 3)]
 
 
 def _run(P, E, a, b, **kw):
