@@ -167,7 +167,8 @@ def build_problem(name, dev, lddp, world, rank, tile_rows=0):
         comm = lddp.lddp_comm_create(plan.handle, world, rank)
         handles = [None] * world
         dist.all_gather_object(handles, lddp.lddp_comm_handle(comm))
-        lddp.lddp_comm_connect(comm, handles[rank + 1] if rank + 1 < world else None)
+        lddp.lddp_comm_connect(comm, handles[rank + 1] if rank + 1 < world else None,
+                               handles[rank - 1] if rank > 0 else None)
         dist.barrier()
     return {"cfg": cfg, "x": x, "plan": plan, "t": t, "comm": comm, "h2d": h2d, "outs": outs}
 

@@ -40,7 +40,7 @@
 extern "C" {
 #endif
 
-#define LDDP_ABI_VERSION 1
+#define LDDP_ABI_VERSION 2
 
 typedef enum {
     LDDP_OK = 0,
@@ -209,23 +209,38 @@ lddp_status lddp_traceback(lddp_plan_t plan, const lddp_inputs* in, const void* 
 lddp_status lddp_status_check(lddp_plan_t plan, void* workspace, void* stream);
 
 /* ---- multi-GPU column strips (one process per GPU) -------------------------------------------
- * Rank g of P owns columns [floor(g*cols/P), floor((g+1)*cols/P)) of every row.  Each rank's
- * persistent kernel stores the right column of every finished row strip straight into rank
- * g+1's receive window over NVLink (peer stores + a release flag; one-way, Table II [L265-L274]
- * anti-diagonal row), and waits on its own window for rank g-1's column.  Supported for the
- * anti-diagonal category (LCS, Levenshtein, DTW) in this build.
- *   lddp_comm_create   allocates this rank's receive window on the plan's device.
- *   lddp_comm_handle   exports it (CUDA IPC handle, LDDP_COMM_HANDLE_BYTES) for rank g-1.
- *   lddp_comm_connect  opens rank g+1's window from its handle (NULL on the last rank).
+ * Rank g of P owns columns [floor(g*cols/P), floor((g+1)*cols/P)) of every row
+ * (lddp_multi_partition).  Each rank's persistent kernel stores the right column of every
+ * finished row strip straight into rank g+1's receive window over NVLink (peer stores + a
+ * system-scope release flag per strip: the one-way boundary transfer of Table II's
+ * anti-diagonal row [L265-L274], [L164]) and reads rank g-1's column from its own window.
+ * Supported for the anti-diagonal category (LCS, Levenshtein, DTW) in this build.
+ *
+ * Window of rank g (device memory of rank g), two slots selected by fill parity so that fill
+ * k+1 can start on rank g-1 while rank g is still reading fill k:
+ *   ack[2][S]       written by rank g+1: fill epoch whose strip s it has finished reading
+ *   flag[2][S]      written by rank g-1: (epoch << 32) | 1 once strip s's column is in
+ *   value[2][m + 1] written by rank g-1: its right column, index i + 1 for row i
+ * A producer reuses slot k & 1 for strip s only after the consumer acknowledged fill k-2 for
+ * strips s and s+1 (strip s+1 also reads strip s's last row); a consumer accepts a flag only if it
+ * equals this fill's epoch.  Every wait is bounded by the device watchdog (LDDP_ERR_TIMEOUT).
+ *   lddp_comm_create   allocates this rank's window on the plan's device (zeroed).
+ *   lddp_comm_handle   exports it (CUDA IPC handle, LDDP_COMM_HANDLE_BYTES).
+ *   lddp_comm_connect  opens rank g+1's and rank g-1's windows from their handles (NULL at the
+ *                      ends of the chain).  Handles travel over any process group (the
+ *                      torch.distributed gloo / NCCL object collectives in bench.py and tests).
  *   lddp_comm_connect_local   in-process alternative (ranks on the same or peer devices).
- * lddp_fill_multi: every rank calls it with the whole a / b (rows / cols of the full problem)
- * and full-size output buffers; rank g writes last_row[c0:c1) and, on the last rank only,
- * score and last_col. */
+ * lddp_fill_multi: every rank calls it once per fill, in the same order (the k-th call on each
+ * rank is fill k), with the whole a / b (rows / cols of the full problem) and full-size output
+ * buffers; rank g writes last_row[c0:c1) and, on the last rank only, score and last_col.  Fills
+ * only enqueue: ranks may run ahead of each other by up to one fill. */
 #define LDDP_COMM_HANDLE_BYTES 64
+/* Columns [c0, c1) of rank `rank` of `nranks` for a problem with `cols` columns (host only). */
+lddp_status lddp_multi_partition(int64_t cols, int32_t nranks, int32_t rank, int64_t* c0, int64_t* c1);
 lddp_status lddp_comm_create(lddp_plan_t plan, int32_t nranks, int32_t rank, lddp_comm_t* comm);
 lddp_status lddp_comm_handle(lddp_comm_t comm, uint8_t handle[LDDP_COMM_HANDLE_BYTES]);
-lddp_status lddp_comm_connect(lddp_comm_t comm, const uint8_t next_handle[LDDP_COMM_HANDLE_BYTES]);
-lddp_status lddp_comm_connect_local(lddp_comm_t comm, lddp_comm_t next);
+lddp_status lddp_comm_connect(lddp_comm_t comm, const uint8_t* next_handle, const uint8_t* prev_handle);
+lddp_status lddp_comm_connect_local(lddp_comm_t comm, lddp_comm_t next, lddp_comm_t prev);
 lddp_status lddp_comm_destroy(lddp_comm_t comm);
 lddp_status lddp_fill_multi(lddp_plan_t plan, const lddp_inputs* in, const lddp_outputs* out,
                             void* workspace, lddp_comm_t comm, void* stream);

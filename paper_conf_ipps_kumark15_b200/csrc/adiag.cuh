@@ -478,10 +478,8 @@ __global__ void __launch_bounds__(W * 32, 1) adiag_kernel(const FillParams p) {
 
     AW aw;
     bool ok = true;
-    if (p.lcol_in != nullptr) {   // multi-GPU: rank g-1's right column of this (and the previous) strip
-      ok = wait_flag<true>(p.lflag_in + s, (p.wepoch << 32) | 1u, ctl, p.timeout_ns);
-      if (ok && s > 0 && wid == 0) ok = wait_flag<true>(p.lflag_in + s - 1, (p.wepoch << 32) | 1u, ctl, p.timeout_ns);
-    }
+    // multi-GPU: rank g-1's right column of this strip and the previous strip's last row
+    if (p.lcol_in != nullptr) ok = window_consume_wait(p, s, ctl);
     aw.irow0 = wtop + (int64_t)lane * R;
 #pragma unroll
     for (int r = 0; r < R; ++r) {
@@ -497,6 +495,10 @@ __global__ void __launch_bounds__(W * 32, 1) adiag_kernel(const FillParams p) {
     for (int d = 0; d <= E; ++d) aw.fifo[d] = T(0);
     // lane 0's UL at column 0: the row above the warp at column -1 (received "before" step -E)
     if (lane == 0) aw.fifo[0] = aw.leftval(p, wtop - 1);
+    if (p.lcol_in != nullptr) {   // every left value of the strip is in registers: release the slot
+      __syncthreads();
+      if (threadIdx.x == 0 && ok) window_consume_ack(p, s);
+    }
     aw.cring = cring[wid];
     aw.one = ad_ld_smem_i32(&one_sh);   // a volatile load: ptxas cannot rematerialise it per use
     aw.small = false;
@@ -629,7 +631,15 @@ __global__ void __launch_bounds__(W * 32, 1) adiag_kernel(const FillParams p) {
       tr[4] = (uint64_t)wait_bp;
       tr[5] = (uint64_t)blockIdx.x;
     }
-    // right column of every row: last_col output, rank g+1's window, the score
+    // right column of every row: last_col output, rank g+1's window (once rank g+1 has released
+    // this slot), the score
+    if (p.rcol_out != nullptr) {
+      __shared__ int pw_ok;
+      __syncthreads();
+      if (threadIdx.x == 0) pw_ok = ok && window_produce_wait(p, s, ctl);
+      __syncthreads();
+      ok = ok && pw_ok;
+    }
     if (ok) {
 #pragma unroll
       for (int r = 0; r < R; ++r) {

@@ -21,10 +21,10 @@
 //    selector per column (A's code, B's code, zero bytes between), so
 //    m = PRMT(tabA[p], tabB[p], sel) = [a_A = b_cA] + [a_B = b_cB] << 16.
 //    Warps whose rows use more than 4 characters take a table path (per-warp match table).
-//  * Values are RELATIVE to a warp-uniform base (absolute = relative + base), rebased every
-//    chunk: every value a warp holds lies within 381 of its lane 0 (|LCS(i,j) - LCS(i',j')| <=
-//    |i-i'| + |j-j'| over 192 rows and 189 columns), so 16 bits hold them; all handoffs and
-//    outputs are absolute 32-bit.
+//  * Values are RELATIVE to a warp-uniform base (absolute = relative + base), rebased every 8
+//    chunks: every value a warp holds lies within 64P + 64E + 2 of its lane 0 (|LCS(i,j) -
+//    LCS(i',j')| <= |i-i'| + |j-j'| over the strip's 64P rows and 64E columns of lane lag), so
+//    16 bits hold them (rebase()); all handoffs and outputs are absolute 32-bit.
 //  * Boundary columns without per-column selects: before column 0 every lane sweeps "columns"
 //    that match nothing, starting from the left boundary values; for LCS max(U, L, UL) there
 //    keeps every row at its left value (the left column is non-decreasing downwards), so column
@@ -200,10 +200,13 @@ struct L16Warp {
     }
   }
 
-  // Keep relative values small: subtract K = (lane 0's A row 0) - 512 from every register.
+  // Keep relative values small: subtract K = (lane 0's A row 0) - 4096 from every register.
+  // Every value the warp holds is >= v0 - (64P rows + 64E columns + 2 steps of fifo age) >
+  // v0 - 4096 (P, E <= 8), and <= v0 + 64P + 8 chunks of growth < 8192: 16 bits suffice.
   __device__ __forceinline__ void rebase() {
+    static_assert(64 * P + 64 * E + 64 <= 4096, "rebase margin");
     const int32_t v0 = (int32_t)(__shfl_sync(0xffffffffu, h[0], 0) & 0xFFFFu);
-    const int32_t K = v0 > 1024 ? v0 - 512 : 0;
+    const int32_t K = v0 > 8192 ? v0 - 4096 : 0;
     if (K == 0) return;   // warp-uniform
     const uint32_t nk = (uint32_t)(0x10000 - K) & 0xFFFFu;
     const uint32_t nk2 = nk | (nk << 16);
@@ -220,8 +223,10 @@ struct L16Warp {
   __device__ __forceinline__ void chunk(const int lane, const int k, const int NQ, const Links& lk, const int w0) {
     const int lane_off = lane * E;
     // chunk k's top row (relative) -> shared memory; lane 31 injects it one group ahead.  Past
-    // the last chunk any value <= the rows' own keeps them constant: 0 (relative values are >= 0)
-    lk.tstg[lane] = k < NQ ? max((int32_t)(uint32_t)tp - base, 0) : 0;
+    // the last chunk (k >= NQ) tp keeps chunk NQ-1's pair: a top value within 32 columns of
+    // column n-1, <= the rows' own past-the-end values (they stay constant) and close enough to
+    // them to survive later rebases (a constant 0 would wrap below the rebased range)
+    lk.tstg[lane] = max((int32_t)(uint32_t)tp - base, 0);
     __syncwarp();
     uint32_t injq[8];
     {
@@ -397,10 +402,8 @@ __global__ void __launch_bounds__(32 * WPC, 1) lcs16_kernel(const FillParams p) 
 
     LW lw;
     bool ok = true;
-    if (p.lcol_in != nullptr) {   // multi-GPU: rank g-1's right column of this (and the previous) strip
-      ok = wait_flag<true>(p.lflag_in + s, (p.wepoch << 32) | 1u, ctl, p.timeout_ns);
-      if (ok && s > 0) ok = wait_flag<true>(p.lflag_in + s - 1, (p.wepoch << 32) | 1u, ctl, p.timeout_ns);
-    }
+    // multi-GPU: rank g-1's right column of this strip and the previous strip's last row
+    if (p.lcol_in != nullptr) ok = window_consume_wait(p, s, ctl);
     // rows of this lane: A = top + lane*P + q, B = top + 32P + lane*P + q
     const int64_t rowA = top + (int64_t)lane * P, rowB = rowA + 32 * P;
     int32_t chA[P], chB[P];
@@ -419,6 +422,10 @@ __global__ void __launch_bounds__(32 * WPC, 1) lcs16_kernel(const FillParams p) 
 #pragma unroll
     for (int d = 0; d < E; ++d) lw.fifo[d] = up;
     lw.U0p = up;
+    if (p.lcol_in != nullptr) {   // every left value of the strip is in registers: release the slot
+      __syncwarp();
+      if (lane == 0 && ok) window_consume_ack(p, s);
+    }
     lw.one = ad_ld_smem_i32(&one_sh[wid]);
     lw.ssel = lane == 31 ? 0x1054u : 0x3210u;
     lw.ring = ring;
@@ -523,7 +530,13 @@ __global__ void __launch_bounds__(32 * WPC, 1) lcs16_kernel(const FillParams p) 
       tr[6] = 0;
       tr[7] = 0;
     }
-    // right column = the final registers (rows keep their column n-1 value past the end)
+    // right column = the final registers (rows keep their column n-1 value past the end); into
+    // rank g+1's window once rank g+1 has released this slot
+    if (p.rcol_out != nullptr) {
+      int pw = 0;
+      if (lane == 0) pw = ok && window_produce_wait(p, s, ctl);
+      ok = __shfl_sync(0xffffffffu, pw, 0) != 0;
+    }
     if (ok) {
 #pragma unroll
       for (int q = 0; q < P; ++q) {

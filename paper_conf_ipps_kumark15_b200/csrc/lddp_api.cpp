@@ -224,14 +224,18 @@ struct lddp_plan_s {
   size_t stage_bytes[6];
 };
 
+// Multi-GPU receive window (lddp.h): [ack 2 x S u64][flag 2 x S u64][value 2 x (m + 1) x 4 B]
 struct lddp_comm_s {
   lddp_plan_t plan;
   int nranks, rank, device;
-  void* window;          // [flags: nstrips u64][values: rows x 4 B]
+  void* window;          // this rank's window (device memory of this rank)
   size_t win_bytes;
-  void* peer;            // rank+1's window (IPC-opened or in-process)
-  bool peer_ipc;
-  uint64_t fills;
+  size_t off_flag, off_val;
+  int64_t nstrips, rows;
+  void* next;            // rank+1's window (IPC-opened or in-process), NULL on the last rank
+  void* prev;            // rank-1's window, NULL on rank 0
+  bool next_ipc, prev_ipc;
+  uint64_t fills;        // fill epoch k of the next lddp_fill_multi (rank-consistent call order)
 };
 
 namespace {
@@ -523,6 +527,12 @@ lddp_status lddp_plan(const lddp_desc* desc, lddp_plan_t* out) {
       pl->E = env_int("LDDP_L16_E", 2);
       pl->W = 1;
       pl->SIG = 0;
+      if (!lddp::lcs16_compiled(pl->R, pl->E)) {   // nearest compiled P for this E (tile_rows hint)
+        int best = -1;
+        for (int P = 1; P <= 8; ++P)
+          if (lddp::lcs16_compiled(P, pl->E) && (best < 0 || std::abs(P - pl->R) < std::abs(best - pl->R))) best = P;
+        if (best > 0) pl->R = best;
+      }
       if (!lddp::lcs16_compiled(pl->R, pl->E)) {
         const int P = pl->R, E = pl->E;
         delete pl;
@@ -857,11 +867,19 @@ lddp_status lddp_status_check(lddp_plan_t pl, void* ws, void* stream) {
 }
 
 // ------------------------------------------------------------------------------ multi-GPU
+lddp_status lddp_multi_partition(int64_t cols, int32_t nranks, int32_t rank, int64_t* c0, int64_t* c1) {
+  if (c0 == nullptr || c1 == nullptr) return fail(LDDP_ERR_INVALID_ARG, "NULL argument");
+  if (cols < 0 || nranks < 1 || rank < 0 || rank >= nranks) return fail(LDDP_ERR_INVALID_ARG, "bad partition request");
+  *c0 = (int64_t)rank * cols / nranks;
+  *c1 = (int64_t)(rank + 1) * cols / nranks;
+  return LDDP_OK;
+}
+
 lddp_status lddp_comm_create(lddp_plan_t pl, int32_t nranks, int32_t rank, lddp_comm_t* out) {
   if (pl == nullptr || out == nullptr) return fail(LDDP_ERR_INVALID_ARG, "NULL argument");
   if (nranks < 1 || rank < 0 || rank >= nranks) return fail(LDDP_ERR_INVALID_ARG, "bad rank %d / %d", rank, nranks);
-  if ((pl->kind != 0 && pl->kind != 3 && pl->kind != 4) || pl->desc.category != LDDP_CAT_ANTI_DIAGONAL)
-    return fail(LDDP_ERR_UNSUPPORTED, "multi-GPU column strips: anti-diagonal category only in this build");
+  if ((pl->kind != 3 && pl->kind != 4) || pl->desc.category != LDDP_CAT_ANTI_DIAGONAL)
+    return fail(LDDP_ERR_UNSUPPORTED, "multi-GPU column strips: anti-diagonal LCS / Levenshtein / DTW (no TABLE)");
   if (pl->desc.cols < nranks) return fail(LDDP_ERR_SHAPE, "cols < nranks");
   DeviceGuard dg(pl->desc.device);
   lddp_comm_s* c = new (std::nothrow) lddp_comm_s();
@@ -870,13 +888,19 @@ lddp_status lddp_comm_create(lddp_plan_t pl, int32_t nranks, int32_t rank, lddp_
   c->nranks = nranks;
   c->rank = rank;
   c->device = pl->desc.device;
-  c->win_bytes = align_up((size_t)std::max(pl->nstrips, 1) * 8, 256) + (size_t)std::max<int64_t>(pl->desc.rows, 1) * 4;
+  // strips of the widest geometry this plan can launch (lcs16 falls back to 192-row strips)
+  c->nstrips = std::max<int64_t>(std::max<int64_t>(pl->nstrips, (pl->desc.rows + 191) / 192), 1);
+  c->rows = pl->desc.rows;
+  c->off_flag = align_up((size_t)2 * c->nstrips * 8, 256);
+  c->off_val = c->off_flag + align_up((size_t)2 * c->nstrips * 8, 256);
+  c->win_bytes = c->off_val + (size_t)2 * (c->rows + 1) * 4;
   cudaError_t e = cudaMalloc(&c->window, c->win_bytes);
   if (e == cudaSuccess) e = cudaMemset(c->window, 0, c->win_bytes);
   if (e != cudaSuccess) {
     delete c;
     return cuda_fail(e, "window allocation");
   }
+  c->fills = 0;
   *out = c;
   return LDDP_OK;
 }
@@ -893,48 +917,74 @@ lddp_status lddp_comm_handle(lddp_comm_t c, uint8_t handle[LDDP_COMM_HANDLE_BYTE
   return LDDP_OK;
 }
 
-lddp_status lddp_comm_connect(lddp_comm_t c, const uint8_t next_handle[LDDP_COMM_HANDLE_BYTES]) {
-  if (c == nullptr) return fail(LDDP_ERR_INVALID_ARG, "comm is NULL");
-  if (c->rank == c->nranks - 1 || next_handle == nullptr) {
-    c->peer = nullptr;
-    return LDDP_OK;
-  }
-  DeviceGuard dg(c->device);
+namespace {
+lddp_status open_ipc(const uint8_t* handle, void** out) {
   cudaIpcMemHandle_t h;
-  memcpy(&h, next_handle, sizeof h);
+  memcpy(&h, handle, sizeof h);
   void* p = nullptr;
   cudaError_t e = cudaIpcOpenMemHandle(&p, h, cudaIpcMemLazyEnablePeerAccess);
   if (e != cudaSuccess) return fail(LDDP_ERR_COMM, "cudaIpcOpenMemHandle: %s", cudaGetErrorString(e));
-  c->peer = p;
-  c->peer_ipc = true;
+  *out = p;
+  return LDDP_OK;
+}
+lddp_status enable_peer(int dev, int peer) {
+  if (peer == dev) return LDDP_OK;
+  DeviceGuard dg(dev);
+  int ok = 0;
+  cudaDeviceCanAccessPeer(&ok, dev, peer);
+  if (!ok) return fail(LDDP_ERR_COMM, "device %d cannot access peer %d", dev, peer);
+  cudaError_t e = cudaDeviceEnablePeerAccess(peer, 0);
+  if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled)
+    return fail(LDDP_ERR_COMM, "cudaDeviceEnablePeerAccess: %s", cudaGetErrorString(e));
+  cudaGetLastError();
+  return LDDP_OK;
+}
+}  // namespace
+
+lddp_status lddp_comm_connect(lddp_comm_t c, const uint8_t* next_handle, const uint8_t* prev_handle) {
+  if (c == nullptr) return fail(LDDP_ERR_INVALID_ARG, "comm is NULL");
+  if ((c->rank < c->nranks - 1) != (next_handle != nullptr))
+    return fail(LDDP_ERR_INVALID_ARG, "rank %d of %d: next handle must be given iff a next rank exists", c->rank, c->nranks);
+  if ((c->rank > 0) != (prev_handle != nullptr))
+    return fail(LDDP_ERR_INVALID_ARG, "rank %d: previous handle must be given iff a previous rank exists", c->rank);
+  DeviceGuard dg(c->device);
+  if (next_handle != nullptr) {
+    lddp_status st = open_ipc(next_handle, &c->next);
+    if (st != LDDP_OK) return st;
+    c->next_ipc = true;
+  }
+  if (prev_handle != nullptr) {
+    lddp_status st = open_ipc(prev_handle, &c->prev);
+    if (st != LDDP_OK) return st;
+    c->prev_ipc = true;
+  }
   return LDDP_OK;
 }
 
-lddp_status lddp_comm_connect_local(lddp_comm_t c, lddp_comm_t next) {
+lddp_status lddp_comm_connect_local(lddp_comm_t c, lddp_comm_t next, lddp_comm_t prev) {
   if (c == nullptr) return fail(LDDP_ERR_INVALID_ARG, "comm is NULL");
-  if (next == nullptr) {
-    c->peer = nullptr;
-    return LDDP_OK;
+  if ((c->rank < c->nranks - 1) != (next != nullptr) || (c->rank > 0) != (prev != nullptr))
+    return fail(LDDP_ERR_INVALID_ARG, "rank %d of %d: neighbours must be given iff they exist", c->rank, c->nranks);
+  if (next != nullptr) {
+    lddp_status st = enable_peer(c->device, next->device);
+    if (st != LDDP_OK) return st;
+    c->next = next->window;
+    c->next_ipc = false;
   }
-  if (next->device != c->device) {
-    DeviceGuard dg(c->device);
-    int ok = 0;
-    cudaDeviceCanAccessPeer(&ok, c->device, next->device);
-    if (!ok) return fail(LDDP_ERR_COMM, "device %d cannot access peer %d", c->device, next->device);
-    cudaError_t e = cudaDeviceEnablePeerAccess(next->device, 0);
-    if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled)
-      return fail(LDDP_ERR_COMM, "cudaDeviceEnablePeerAccess: %s", cudaGetErrorString(e));
-    cudaGetLastError();
+  if (prev != nullptr) {
+    lddp_status st = enable_peer(c->device, prev->device);
+    if (st != LDDP_OK) return st;
+    c->prev = prev->window;
+    c->prev_ipc = false;
   }
-  c->peer = next->window;
-  c->peer_ipc = false;
   return LDDP_OK;
 }
 
 lddp_status lddp_comm_destroy(lddp_comm_t c) {
   if (c == nullptr) return LDDP_OK;
   DeviceGuard dg(c->device);
-  if (c->peer_ipc && c->peer) cudaIpcCloseMemHandle(c->peer);
+  if (c->next_ipc && c->next) cudaIpcCloseMemHandle(c->next);
+  if (c->prev_ipc && c->prev) cudaIpcCloseMemHandle(c->prev);
   if (c->window) cudaFree(c->window);
   delete c;
   return LDDP_OK;
@@ -969,8 +1019,11 @@ lddp_status lddp_fill_multi(lddp_plan_t pl, const lddp_inputs* in, const lddp_ou
     if (c->plan != pl) return fail(LDDP_ERR_INVALID_ARG, "comm was created for another plan");
     lddp_status st = check_inputs(pl, in, out);
     if (st != LDDP_OK) return st;
-    if (c->rank < c->nranks - 1 && c->peer == nullptr)
+    if (c->rank < c->nranks - 1 && c->next == nullptr)
       return fail(LDDP_ERR_COMM, "rank %d is not connected to rank %d", c->rank, c->rank + 1);
+    if (c->rank > 0 && c->prev == nullptr)
+      return fail(LDDP_ERR_COMM, "rank %d is not connected to rank %d", c->rank, c->rank - 1);
+    if (pl->desc.outputs & LDDP_OUT_TABLE) return fail(LDDP_ERR_UNSUPPORTED, "TABLE output is not supported by lddp_fill_multi");
     DeviceGuard dg(pl->desc.device);
     cudaStream_t s = (cudaStream_t)stream;
     const lddp_desc& d = pl->desc;
@@ -978,39 +1031,37 @@ lddp_status lddp_fill_multi(lddp_plan_t pl, const lddp_inputs* in, const lddp_ou
     st = ensure_own_ws(pl, &ws, s);
     if (st != LDDP_OK) return st;
     const int64_t n = d.cols;
-    const int64_t c0 = (int64_t)c->rank * n / c->nranks;
-    const int64_t c1 = (int64_t)(c->rank + 1) * n / c->nranks;
+    int64_t c0 = 0, c1 = 0;
+    lddp_multi_partition(n, c->nranks, c->rank, &c0, &c1);
     FillParams p;
     fill_common(pl, in, out, ws, p);
     p.cols = (int32_t)(c1 - c0);
     p.col0 = (int32_t)c0;
     p.cols_total = (int32_t)n;
-    if (pl->kind == 3 || pl->kind == 4) {
-      p.nchunks = (int)((p.cols + 31) / 32);
-      p.bnd_stride = (int64_t)std::max(p.nchunks, 1) * 32;
-    } else {
-      p.nchunks = (int)((p.cols + 33 + 31) / 32);
-      p.bnd_stride = (int64_t)p.nchunks * 32;
-    }
+    p.nchunks = (int)((p.cols + 31) / 32);
+    p.bnd_stride = (int64_t)std::max(p.nchunks, 1) * 32;
     const bool last = c->rank == c->nranks - 1;
     p.is_last_rank = last ? 1 : 0;
     if (p.last_row) p.last_row = static_cast<char*>(p.last_row) + c0 * cell_bytes(d.func);
     if (!last) {
       p.score = nullptr;
       p.last_col = nullptr;
-      p.table = nullptr;
     }
-    if (p.table) return fail(LDDP_ERR_UNSUPPORTED, "TABLE output is not supported by lddp_fill_multi");
-    const size_t flags_bytes = align_up((size_t)std::max(pl->nstrips, 1) * 8, 256);
+    // fill epoch k (1, 2, ...) and its window slot k & 1
     c->fills += 1;
     p.wepoch = c->fills;
+    const int slot = (int)(p.wepoch & 1);
+    const size_t val_slot = (size_t)slot * (c->rows + 1) * 4 + 4;   // element 0 = row -1
+    auto win = [&](void* base, size_t off) { return reinterpret_cast<char*>(base) + off; };
     if (c->rank > 0) {
-      p.lflag_in = reinterpret_cast<const uint64_t*>(c->window);
-      p.lcol_in = static_cast<const char*>(c->window) + flags_bytes;
+      p.lflag_in = reinterpret_cast<const uint64_t*>(win(c->window, c->off_flag)) + slot * c->nstrips;
+      p.lcol_in = win(c->window, c->off_val + val_slot);
+      p.ack_out = reinterpret_cast<uint64_t*>(win(c->prev, 0)) + slot * c->nstrips;
     }
     if (!last) {
-      p.rflag_out = reinterpret_cast<uint64_t*>(c->peer);
-      p.rcol_out = static_cast<char*>(c->peer) + flags_bytes;
+      p.ack_in = reinterpret_cast<const uint64_t*>(win(c->window, 0)) + slot * c->nstrips;
+      p.rflag_out = reinterpret_cast<uint64_t*>(win(c->next, c->off_flag)) + slot * c->nstrips;
+      p.rcol_out = win(c->next, c->off_val + val_slot);
     }
     return launch(pl, p, s);
   } catch (...) {

@@ -42,10 +42,12 @@ struct FillParams {
   int32_t block_cols;       // columns owned per CTA
   int32_t halo;             // trapezoid halo (= band rows)
   int32_t nblocks;          // column blocks
-  // multi-GPU window (left boundary in, right column out)
-  const void* lcol_in;      // my window: rows values of rank g-1's right column
+  // multi-GPU window (left boundary in, right column out), this fill's slot (lddp.h)
+  const void* lcol_in;      // my window: rank g-1's right column, element i = row i (i >= -1)
   const uint64_t* lflag_in; // my window flags, one per strip
-  void* rcol_out;           // rank g+1's window (peer pointer) or NULL
+  uint64_t* ack_out;        // rank g-1's window acks (peer pointer): strip s read by me
+  const uint64_t* ack_in;   // my window acks (written by rank g+1)
+  void* rcol_out;           // rank g+1's window values (peer pointer), element i = row i, or NULL
   uint64_t* rflag_out;      // rank g+1's window flags (peer pointer) or NULL
   // debug trace (env LDDP_TRACE): globaltimer stamps per (strip, warp, chunk), or NULL
   uint64_t* trace;

@@ -171,6 +171,46 @@ __device__ __forceinline__ bool wait_flag(const uint64_t* flag, uint64_t target,
   }
 }
 
+// Wait until an epoch-tagged flag EQUALS `target` (multi-GPU window slots are reused every
+// other fill: an older epoch must not pass).
+__device__ __forceinline__ bool wait_flag_eq_sys(const uint64_t* flag, uint64_t target, Control* ctl,
+                                                 uint64_t timeout_ns) {
+  Watch<true> w;
+  while (true) {
+    if (ld_acquire_sys(flag) == target) return true;
+    if (!w.tick(ctl, timeout_ns)) return false;
+  }
+}
+
+// ---- multi-GPU receive window protocol (lddp.h "multi-GPU column strips"); wepoch = fill k
+// Consumer, before reading strip s's left column (rows top_s - 1 .. top_s + SH - 1): the strip's
+// flag and the previous strip's (its last row) must carry this fill's epoch.
+template <class Params>
+__device__ __forceinline__ bool window_consume_wait(const Params& p, int s, Control* ctl) {
+  const uint64_t tag = (p.wepoch << 32) | 1u;
+  if (!wait_flag_eq_sys(p.lflag_in + s, tag, ctl, p.timeout_ns)) return false;
+  return s == 0 || wait_flag_eq_sys(p.lflag_in + s - 1, tag, ctl, p.timeout_ns);
+}
+// Consumer, after every thread of the strip has read its left values (caller synchronises):
+// tell rank g-1 that slot (k & 1) of strip s may be reused.
+template <class Params>
+__device__ __forceinline__ void window_consume_ack(const Params& p, int s) {
+  if (p.ack_out != nullptr) st_release_sys(p.ack_out + s, p.wepoch);
+}
+// Producer, before storing strip s's right column into rank g+1's slot (k & 1): rank g+1 has
+// finished reading fill k-2 there (strips s and s+1, which reads strip s's last row).
+template <class Params>
+__device__ __forceinline__ bool window_produce_wait(const Params& p, int s, Control* ctl) {
+  if (p.wepoch <= 2) return true;
+  const uint64_t need = p.wepoch - 2;
+  for (int t = s; t <= s + 1 && t < p.nstrips; ++t) {
+    Watch<true> w;
+    while (ld_acquire_sys(p.ack_in + t) < need)
+      if (!w.tick(ctl, p.timeout_ns)) return false;
+  }
+  return true;
+}
+
 // Acquire pattern without an L1 invalidation per poll: relaxed polls, then one acq_rel fence
 // once the released value is observed.  Returns the observed flag in `seen`.
 __device__ __forceinline__ bool wait_flag_relaxed(const uint64_t* flag, uint64_t target, Control* ctl,

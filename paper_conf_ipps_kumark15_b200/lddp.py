@@ -79,8 +79,10 @@ _SIGS = {
     "lddp_status_check": (ctypes.c_int, [_P, _P, _P]),
     "lddp_comm_create": (ctypes.c_int, [_P, ctypes.c_int32, ctypes.c_int32, ctypes.POINTER(_P)]),
     "lddp_comm_handle": (ctypes.c_int, [_P, ctypes.c_char_p]),
-    "lddp_comm_connect": (ctypes.c_int, [_P, ctypes.c_char_p]),
-    "lddp_comm_connect_local": (ctypes.c_int, [_P, _P]),
+    "lddp_comm_connect": (ctypes.c_int, [_P, ctypes.c_char_p, ctypes.c_char_p]),
+    "lddp_comm_connect_local": (ctypes.c_int, [_P, _P, _P]),
+    "lddp_multi_partition": (ctypes.c_int, [ctypes.c_int64, ctypes.c_int32, ctypes.c_int32,
+                                            ctypes.POINTER(ctypes.c_int64), ctypes.POINTER(ctypes.c_int64)]),
     "lddp_comm_destroy": (ctypes.c_int, [_P]),
     "lddp_fill_multi": (ctypes.c_int, [_P, ctypes.POINTER(lddp_inputs), ctypes.POINTER(lddp_outputs), _P, _P, _P]),
     "lddp_traceback": (ctypes.c_int, [_P, ctypes.POINTER(lddp_inputs), _P, ctypes.c_int64, _P, _P, _P, _P]),
@@ -178,12 +180,22 @@ def lddp_comm_handle(comm) -> bytes:
     return buf.raw
 
 
-def lddp_comm_connect(comm, next_handle) -> None:
-    _check(_lib.lddp_comm_connect(comm, next_handle), "lddp_comm_connect")
+def lddp_comm_connect(comm, next_handle, prev_handle=None) -> None:
+    """next_handle: rank g+1's window handle (None on the last rank); prev_handle: rank g-1's
+    (None on rank 0)."""
+    _check(_lib.lddp_comm_connect(comm, next_handle, prev_handle), "lddp_comm_connect")
 
 
-def lddp_comm_connect_local(comm, next_comm) -> None:
-    _check(_lib.lddp_comm_connect_local(comm, next_comm), "lddp_comm_connect_local")
+def lddp_comm_connect_local(comm, next_comm, prev_comm=None) -> None:
+    _check(_lib.lddp_comm_connect_local(comm, next_comm, prev_comm), "lddp_comm_connect_local")
+
+
+def lddp_multi_partition(cols: int, nranks: int, rank: int):
+    """Columns [c0, c1) rank `rank` of `nranks` owns (host only, no GPU needed)."""
+    c0, c1 = ctypes.c_int64(), ctypes.c_int64()
+    _check(_lib.lddp_multi_partition(cols, nranks, rank, ctypes.byref(c0), ctypes.byref(c1)),
+           "lddp_multi_partition")
+    return c0.value, c1.value
 
 
 def lddp_comm_destroy(comm) -> None:

@@ -40,7 +40,7 @@ def test_header_symbols_exported(lddp):
 
 
 def test_abi_version_and_strings(lddp):
-    assert lddp.lddp_abi_version() == 1
+    assert lddp.lddp_abi_version() == 2
     for st, name in lddp.STATUS_NAMES.items():
         assert lddp._lib.lddp_status_string(st).decode() == name
 

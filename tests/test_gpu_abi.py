@@ -110,10 +110,20 @@ def test_plan_describe_and_workspace(L):
     try:
         import json
         info = json.loads(L.lddp_plan_describe(plan))
-        # sequence f's without TABLE output run the lane-systolic adiag kernel
+        # LCS without TABLE output runs the packed 16x2 kernel: 64 virtual lanes x P row pairs
+        assert info["kernel"] == "lcs16" and info["strips"] >= 1
+        assert info["strip_rows"] == 64 * info["rows_per_lane"]
+        assert L.lddp_plan_workspace_size(plan) > 0
+    finally:
+        L.lddp_plan_destroy(plan)
+    d = L.lddp_desc(rows=5000, cols=3000, category=L.CAT_ANTI_DIAGONAL, func=L.F_LEVENSHTEIN, outputs=L.OUT_SCORE)
+    plan = L.lddp_plan(d)
+    try:
+        import json
+        info = json.loads(L.lddp_plan_describe(plan))
+        # the other sequence f's run the 32-bit lane-systolic adiag kernel
         assert info["kernel"] == "adiag" and info["strips"] >= 1
         assert info["strip_rows"] == 32 * info["warps"] * info["rows_per_lane"]
-        assert L.lddp_plan_workspace_size(plan) > 0
     finally:
         L.lddp_plan_destroy(plan)
     d = L.lddp_desc(rows=500, cols=300, category=L.CAT_ANTI_DIAGONAL, func=L.F_LCS,

@@ -108,3 +108,17 @@ def test_lcs16_small_grid(grid):
     m, n = 192 * 7 + 17, 777
     a, b = inputs.gen_strings(grid, m, n)
     _check(_run(3, 3, a, b, grid_ctas=grid, reps=3), oracle.lcs(a, b))
+
+
+@pytest.mark.parametrize("P,E", GEOMS)
+@pytest.mark.parametrize("alphabet", ["one", "dna"])
+def test_lcs16_rebase_every_geometry(P, E, alphabet):
+    """Values far above the rebase threshold (8192) in every compiled geometry: the relative
+    16-bit encoding is rebased many times per strip, with the widest value spread the geometry
+    allows (one letter: LCS grows by one per column and row)."""
+    m, n = (12001, 13003) if alphabet == "one" else (14000, 15001)
+    if alphabet == "one":
+        a, b = np.full(m, 71, np.uint8), np.full(n, 71, np.uint8)
+    else:
+        a, b = inputs.gen_strings(P * 10 + E, m, n)
+    _check(_run(P, E, a, b), oracle.lcs(a, b))

@@ -1,7 +1,18 @@
-"""Multi-GPU column-strip fill (lddp_fill_multi) exercised on ONE GPU: P virtual ranks, each with
-its own comm window, workspace and stream, chained with lddp_comm_connect_local.  The kernel
-path is the same as across GPUs (peer stores of the strip's right column into rank g+1's window
-+ system-scope release flags); only the pointer is local.  Results must equal the oracle."""
+"""Multi-GPU column-strip fill (lddp_fill_multi) exercised on ONE GPU.
+
+* Loopback: P virtual ranks in one process, each with its own comm window, workspace and stream,
+  chained with lddp_comm_connect_local.  The kernel path is the one used across GPUs (peer stores
+  of each strip's right column into rank g+1's window slot, system-scope flags, consumer acks).
+* Every fill of a test uses DIFFERENT inputs and outputs, and the fills are enqueued rank by rank
+  (all fills of rank 0 before any fill of rank 1, ...), so producers run up to two fills ahead of
+  their consumers: a receive window reused without back-pressure would hand rank g+1 the wrong
+  fill's column.  Each result must equal the oracle.
+* Cross-process: 2-3 processes on the same GPU exchange CUDA IPC window handles over a gloo
+  process group (lddp_comm_handle / lddp_comm_connect), the path bench.py takes across GPUs."""
+import os
+import socket
+import time
+
 import numpy as np
 import pytest
 
@@ -10,38 +21,67 @@ from paper_conf_ipps_kumark15_b200 import inputs
 
 pytestmark = pytest.mark.gpu
 
+REF = {"lcs": oracle.lcs, "levenshtein": oracle.levenshtein, "dtw": oracle.dtw}
 
-def run_loopback(func, a, b, P, grid_per_rank=24, reps=2):
+
+def _inputs(func, seed, m, n):
+    return inputs.gen_walks(seed, m, n) if func == "dtw" else inputs.gen_strings(seed, m, n)
+
+
+def _check(func, got, ref):
+    s, lr, lc = got
+    if func == "dtw":
+        assert np.float32(s).tobytes() == np.float32(ref.score).tobytes()
+        np.testing.assert_array_equal(lr.view(np.int32), ref.last_row.view(np.int32))
+        np.testing.assert_array_equal(lc.view(np.int32), ref.last_col.view(np.int32))
+    else:
+        assert s == ref.score
+        np.testing.assert_array_equal(lr, ref.last_row)
+        np.testing.assert_array_equal(lc, ref.last_col)
+
+
+def run_loopback(func, problems, P, grid_per_rank=16, delay_ranks=0.0, kernel=None):
+    """problems: list of (a, b), one fill each.  Returns [(score, last_row, last_col)]."""
     import torch
 
     from paper_conf_ipps_kumark15_b200 import lddp
 
+    old = os.environ.get("LDDP_KERNEL")
+    if kernel:
+        os.environ["LDDP_KERNEL"] = kernel
     dev = torch.device("cuda:0")
-    m, n = len(a), len(b)
+    m, n = len(problems[0][0]), len(problems[0][1])
     cell = torch.float32 if func == "dtw" else torch.int32
-    plan = lddp.Plan(func, "anti_diagonal", m, n,
-                     lddp.OUT_SCORE | lddp.OUT_LAST_ROW | lddp.OUT_LAST_COL, grid_ctas=grid_per_rank)
+    try:
+        plan = lddp.Plan(func, "anti_diagonal", m, n,
+                         lddp.OUT_SCORE | lddp.OUT_LAST_ROW | lddp.OUT_LAST_COL, grid_ctas=grid_per_rank)
+    finally:
+        if kernel:
+            if old is None:
+                os.environ.pop("LDDP_KERNEL", None)
+            else:
+                os.environ["LDDP_KERNEL"] = old
     comms = [lddp.lddp_comm_create(plan.handle, P, g) for g in range(P)]
     for g in range(P):
-        lddp.lddp_comm_connect_local(comms[g], comms[g + 1] if g + 1 < P else None)
-    ta = torch.from_numpy(np.ascontiguousarray(a)).to(dev)
-    tb = torch.from_numpy(np.ascontiguousarray(b)).to(dev)
-    score = torch.full((1,), -7, dtype=cell, device=dev)
-    last_row = torch.full((n,), -7, dtype=cell, device=dev)
-    last_col = torch.full((m,), -7, dtype=cell, device=dev)
+        lddp.lddp_comm_connect_local(comms[g], comms[g + 1] if g + 1 < P else None, comms[g - 1] if g > 0 else None)
+    tens = [(torch.from_numpy(np.ascontiguousarray(a)).to(dev), torch.from_numpy(np.ascontiguousarray(b)).to(dev))
+            for a, b in problems]
+    outs = [(torch.full((1,), -7, dtype=cell, device=dev), torch.full((n,), -7, dtype=cell, device=dev),
+             torch.full((m,), -7, dtype=cell, device=dev)) for _ in problems]
     wss = [torch.zeros(plan.ws_bytes, dtype=torch.uint8, device=dev) for _ in range(P)]
     streams = [torch.cuda.Stream(dev) for _ in range(P)]
     torch.cuda.synchronize()
     try:
-        for _ in range(reps):
-            for g in range(P):
-                inp, out = plan.io(a=ta, b=tb, score=score, last_row=last_row, last_col=last_col)
-                lddp.lddp_fill_multi(plan.handle, inp, out, wss[g].data_ptr(), comms[g],
-                                     streams[g].cuda_stream)
-            for g in range(P):
-                lddp.lddp_status_check(plan.handle, wss[g].data_ptr(), streams[g].cuda_stream)
+        for g in range(P):   # rank by rank: rank g enqueues every fill before rank g+1 starts
+            for (ta, tb), (sc, lr, lc) in zip(tens, outs):
+                inp, out = plan.io(a=ta, b=tb, score=sc, last_row=lr, last_col=lc)
+                lddp.lddp_fill_multi(plan.handle, inp, out, wss[g].data_ptr(), comms[g], streams[g].cuda_stream)
+            if delay_ranks:
+                time.sleep(delay_ranks)
+        for g in range(P):
+            lddp.lddp_status_check(plan.handle, wss[g].data_ptr(), streams[g].cuda_stream)
         torch.cuda.synchronize()
-        return score.cpu().numpy()[0], last_row.cpu().numpy(), last_col.cpu().numpy()
+        return [(sc.cpu().numpy()[0], lr.cpu().numpy(), lc.cpu().numpy()) for sc, lr, lc in outs]
     finally:
         for c in comms:
             lddp.lddp_comm_destroy(c)
@@ -51,18 +91,104 @@ def run_loopback(func, a, b, P, grid_per_rank=24, reps=2):
 @pytest.mark.parametrize("P", [2, 3, 4])
 @pytest.mark.parametrize("shape", [(700, 900), (1537, 1000), (2100, 4001)])
 def test_loopback_column_strips(func, P, shape):
+    """Four fills with different inputs, enqueued rank by rank (producers run ahead)."""
     m, n = shape
-    if func == "dtw":
-        a, b = inputs.gen_walks(m + n + P, m, n)
-    else:
-        a, b = inputs.gen_strings(m + n + P, m, n)
-    ref = {"lcs": oracle.lcs, "levenshtein": oracle.levenshtein, "dtw": oracle.dtw}[func](a, b)
-    s, lr, lc = run_loopback(func, a, b, P)
-    if func == "dtw":
-        assert s.tobytes() == np.float32(ref.score).tobytes()
-        np.testing.assert_array_equal(lr.view(np.int32), ref.last_row.view(np.int32))
-        np.testing.assert_array_equal(lc.view(np.int32), ref.last_col.view(np.int32))
-    else:
-        assert s == ref.score
-        np.testing.assert_array_equal(lr, ref.last_row)
-        np.testing.assert_array_equal(lc, ref.last_col)
+    probs = [_inputs(func, 100 * k + m + n + P, m, n) for k in range(4)]
+    for got, (a, b) in zip(run_loopback(func, probs, P), probs):
+        _check(func, got, REF[func](a, b))
+
+
+@pytest.mark.parametrize("kernel", ["adiag", None])
+def test_loopback_back_pressure(kernel):
+    """Rank 1 starts only after rank 0 has enqueued (and started) five fills: rank 0's third fill
+    must wait on the GPU for rank 1's acknowledgement of the first before reusing its window slot."""
+    probs = [_inputs("lcs", 7 * k + 1, 1000, 800) for k in range(5)]
+    for got, (a, b) in zip(run_loopback("lcs", probs, 2, delay_ranks=0.2, kernel=kernel), probs):
+        _check("lcs", got, oracle.lcs(a, b))
+
+
+@pytest.mark.parametrize("P", [2, 3])
+def test_loopback_adiag_dtw_lev(P):
+    """The 32-bit adiag kernel's window path (LCS forced onto it too)."""
+    for func, kernel in (("lcs", "adiag"), ("levenshtein", None), ("dtw", None)):
+        probs = [_inputs(func, 31 * k + P, 1200, 700) for k in range(3)]
+        for got, (a, b) in zip(run_loopback(func, probs, P, kernel=kernel), probs):
+            _check(func, got, REF[func](a, b))
+
+
+# ------------------------------------------------------------------------------ cross-process
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    return port
+
+
+def _ipc_rank(rank, world, port, func, m, n, fills, q):
+    import torch
+    import torch.distributed as dist
+
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    from paper_conf_ipps_kumark15_b200 import inputs as inp_mod
+    from paper_conf_ipps_kumark15_b200 import lddp
+    dev = torch.device("cuda:0")
+    torch.cuda.set_device(dev)
+    cell = torch.float32 if func == "dtw" else torch.int32
+    plan = lddp.Plan(func, "anti_diagonal", m, n, lddp.OUT_SCORE | lddp.OUT_LAST_ROW | lddp.OUT_LAST_COL,
+                     grid_ctas=8)
+    comm = lddp.lddp_comm_create(plan.handle, world, rank)
+    handles = [None] * world
+    dist.all_gather_object(handles, lddp.lddp_comm_handle(comm))
+    lddp.lddp_comm_connect(comm, handles[rank + 1] if rank + 1 < world else None,
+                           handles[rank - 1] if rank > 0 else None)
+    dist.barrier()
+    c0, c1 = lddp.lddp_multi_partition(n, world, rank)
+    res = []
+    bufs = []
+    stream = torch.cuda.current_stream(dev)
+    if rank == 1:
+        time.sleep(0.5)   # rank 0 runs ahead: its later fills must wait for rank 1's acks
+    for k in range(fills):
+        a, b = (inp_mod.gen_walks if func == "dtw" else inp_mod.gen_strings)(1000 + 17 * k, m, n)
+        ta, tb = torch.from_numpy(a).to(dev), torch.from_numpy(b).to(dev)
+        sc = torch.full((1,), -7, dtype=cell, device=dev)
+        lr = torch.full((n,), -7, dtype=cell, device=dev)
+        lc = torch.full((m,), -7, dtype=cell, device=dev)
+        inp, out = plan.io(a=ta, b=tb, score=sc, last_row=lr, last_col=lc)
+        lddp.lddp_fill_multi(plan.handle, inp, out, plan.ws.data_ptr(), comm, stream.cuda_stream)
+        bufs.append((ta, tb, sc, lr, lc))
+    lddp.lddp_status_check(plan.handle, plan.ws.data_ptr(), stream.cuda_stream)
+    for ta, tb, sc, lr, lc in bufs:
+        res.append((float(sc.cpu().numpy()[0]), lr.cpu().numpy()[c0:c1].tolist(),
+                    lc.cpu().numpy().tolist() if rank == world - 1 else None))
+    dist.barrier()
+    lddp.lddp_comm_destroy(comm)
+    q.put((rank, c0, c1, res))
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("func,world", [("lcs", 2), ("lcs", 3), ("dtw", 2)])
+def test_cross_process_ipc(func, world):
+    import torch.multiprocessing as mp
+    m, n, fills = 900, 700, 3
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_ipc_rank, args=(r, world, port, func, m, n, fills, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    parts = sorted([q.get(timeout=300) for _ in range(world)])
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    for k in range(fills):
+        a, b = (inputs.gen_walks if func == "dtw" else inputs.gen_strings)(1000 + 17 * k, m, n)
+        ref = REF[func](a, b)
+        last = np.zeros(n, ref.last_row.dtype)
+        for rank, c0, c1, res in parts:
+            last[c0:c1] = np.asarray(res[k][1], ref.last_row.dtype)
+        score = parts[-1][3][k][0]
+        lcol = np.asarray(parts[-1][3][k][2], ref.last_col.dtype)
+        _check(func, (np.asarray(score, ref.last_row.dtype), last, lcol), ref)

@@ -23,8 +23,8 @@ def test_missing_left_neighbour_times_out():
         plan = lddp.Plan("lcs", "anti_diagonal", 1000, 600, lddp.OUT_SCORE | lddp.OUT_LAST_ROW, grid_ctas=8)
         c0 = lddp.lddp_comm_create(plan.handle, 2, 0)
         c1 = lddp.lddp_comm_create(plan.handle, 2, 1)
-        lddp.lddp_comm_connect_local(c0, c1)
-        lddp.lddp_comm_connect_local(c1, None)
+        lddp.lddp_comm_connect_local(c0, c1, None)
+        lddp.lddp_comm_connect_local(c1, None, c0)
         ta, tb = torch.from_numpy(a).to(dev), torch.from_numpy(b).to(dev)
         score = torch.zeros(1, dtype=torch.int32, device=dev)
         lr = torch.zeros(600, dtype=torch.int32, device=dev)

@@ -1,11 +1,11 @@
 """CPU (gloo) test of the multi-GPU column-strip decomposition used by lddp_fill_multi.
 
-Each process plays one rank: it owns columns [floor(g*n/P), floor((g+1)*n/P)), walks the same
-bottom-aligned row strips as the wavefront kernel (512 rows = 4 warps x 32 lanes x 4 rows),
-receives rank g-1's right column for each strip (torch.distributed recv: the NVLink window
-write of the GPU path) and sends its own right column to rank g+1 once the strip is done --
-the same one-way message order as the kernel (Table II anti-diagonal row, [L265-L274]).  The
-assembled last row / score must equal the monolithic oracle."""
+Each process plays one rank: it owns the columns liblddp.so assigns it (lddp_multi_partition,
+a host-only call of the C ABI), walks bottom-aligned row strips of the lcs16 height (384 rows =
+64 virtual lanes x 6 rows), receives rank g-1's right column for each strip (torch.distributed
+recv: the NVLink window store of the GPU path) and sends its own right column to rank g+1 once
+the strip is done -- the one-way message order of the kernels (Table II anti-diagonal row,
+[L265-L274]).  The assembled last row / score must equal the monolithic oracle."""
 import os
 import socket
 
@@ -15,7 +15,7 @@ import torch
 import torch.distributed as dist
 import torch.multiprocessing as mp
 
-STRIP_ROWS = 4 * 32 * 4
+STRIP_ROWS = 64 * 6
 
 
 def _free_port():
@@ -51,9 +51,9 @@ def _fill_block(a, b, top, left, corner):
 def _rank_main(rank, world, port, m, n, seed, q):
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     dist.init_process_group("gloo", rank=rank, world_size=world)
-    from paper_conf_ipps_kumark15_b200 import inputs
+    from paper_conf_ipps_kumark15_b200 import inputs, lddp
     a, b = inputs.gen_strings(seed, m, n)
-    c0, c1 = rank * n // world, (rank + 1) * n // world
+    c0, c1 = lddp.lddp_multi_partition(n, world, rank)
     top = np.zeros(c1 - c0, np.int64)          # table row 0 (LCS initialisation)
     last_left_bottom = 0                       # corner for the next strip (rank g-1's value)
     for (r0, r1) in _strips(m):
@@ -99,12 +99,18 @@ def test_column_strip_decomposition_gloo(world):
     assert last[-1] == ref.score
 
 
-def test_partition_matches_library_formula():
-    """The C library's rank ranges: floor(g*n/P) .. floor((g+1)*n/P) cover [0, n) exactly."""
-    for n in (1, 7, 100, 100000, 99991):
+def test_library_partition():
+    """lddp_multi_partition (the C library's rank ranges, used by lddp_fill_multi): contiguous,
+    non-empty for cols >= P, covering [0, n) exactly, sizes differing by at most one."""
+    from paper_conf_ipps_kumark15_b200 import lddp
+    for n in (1, 7, 100, 1000, 100000, 99991):
         for P in (1, 2, 3, 4, 8):
             if n < P:
                 continue
-            edges = [g * n // P for g in range(P + 1)]
-            assert edges[0] == 0 and edges[-1] == n
-            assert all(edges[g + 1] > edges[g] for g in range(P))
+            parts = [lddp.lddp_multi_partition(n, P, g) for g in range(P)]
+            assert parts[0][0] == 0 and parts[-1][1] == n
+            assert all(parts[g][1] == parts[g + 1][0] for g in range(P - 1))
+            sizes = [c1 - c0 for c0, c1 in parts]
+            assert min(sizes) >= 1 and max(sizes) - min(sizes) <= 1
+    with pytest.raises(lddp.LddpError):
+        lddp.lddp_multi_partition(10, 2, 2)
