@@ -20,6 +20,7 @@ import argparse
 import hashlib
 import json
 import os
+import subprocess
 import sys
 import threading
 import time
@@ -34,11 +35,14 @@ from configs import CONFIGS  # noqa: E402
 
 PEAKS_FILE = os.path.join(ROOT, "MEASURED_PEAKS.json")
 FALLBACK_PEAKS = {"hbm_gbs": 6650.0, "sm_max_mhz": 1965.0, "_source": "fallback (B200_PROFILING.md)"}
-# Algorithmic work per cell on the binding pipe: LCS = compare + 3-way max on
-# the INT ALU pipe; DTW = subtract + add on the FP32 (FMA) pipe; FS = 4 mul + 5 add on the FMA
-# pipe; min-path = the 4-byte cost read from HBM.
-ALU_OPS_PER_CELL = {"lcs": 2, "levenshtein": 3, "dtw": 2, "fs": 9}
-PIPE_LANES_PER_SM_CLK = 64            # ALU pipe and FMA pipe: 16 lanes/clk per SMSP x 4
+LATENCY_FILE = os.path.join(ROOT, "profiles", "round2_latency.json")   # tools/micro/lat2.cu on B200
+# Algorithmic work per cell, SURVEY.md §8(d) "Algorithmic work per cell": (ops, pipe).  The INT
+# ALU pipe has 64 lanes/clk/SM (16 per SM sub-partition), the FP32 FMA pipe 128.
+WORK = {"lcs": (3, "alu"), "levenshtein": (3, "alu"), "dtw": (3, "fma"), "fs": (11, "fma"),
+        "minpath3": (2, "alu"), "min2plus": (2, "alu"), "diagmaxplus": (2, "alu")}
+LANES = {"alu": 64, "fma": 128}
+# Algorithmic HBM bytes per cell (inputs read once, outputs written once; the table is virtual)
+HBM_PER_CELL = {"fs": 2.0, "minpath3": 4.0, "min2plus": 4.0, "diagmaxplus": 4.0}
 NUM_SMS = 148
 
 
@@ -143,8 +147,10 @@ def build_problem(name, dev, lddp, world, rank, tile_rows=0):
     func, cat = cfg["func"], cfg["category"]
     rows, cols = cfg["rows"], cfg["cols"]
     outs = {"lcs": lddp.OUT_SCORE, "dtw": lddp.OUT_SCORE, "fs": lddp.OUT_TABLE,
-            "minpath3": lddp.OUT_SCORE | lddp.OUT_LAST_ROW}[func]
-    plan = lddp.Plan(func, cat, rows, cols, outs, device=dev.index, tile_rows=tile_rows)
+            "minpath3": lddp.OUT_SCORE | lddp.OUT_LAST_ROW, "min2plus": lddp.OUT_SCORE | lddp.OUT_LAST_ROW,
+            "diagmaxplus": lddp.OUT_LAST_ROW | lddp.OUT_LAST_COL}[func]
+    plan = lddp.Plan(func, cat, rows, cols, outs, device=dev.index, tile_rows=tile_rows,
+                     param_c=cfg.get("param_c", 1))
     t = {}
     h2d = 0
     if "a" in x:
@@ -159,6 +165,8 @@ def build_problem(name, dev, lddp, world, rank, tile_rows=0):
         t["score"] = torch.zeros(1, dtype=cell_dt, device=dev)
     if outs & lddp.OUT_LAST_ROW:
         t["last_row"] = torch.zeros(cols, dtype=cell_dt, device=dev)
+    if outs & lddp.OUT_LAST_COL:
+        t["last_col"] = torch.zeros(rows, dtype=cell_dt, device=dev)
     if outs & lddp.OUT_TABLE:
         t["table"] = torch.zeros((rows, cols), dtype=torch.uint8, device=dev)
     comm = None
@@ -275,6 +283,8 @@ def check_result(name, pb):
             ok &= got["score"] == ref["score"]
     if "last_row_sha256" in ref and "last_row" in t:
         ok &= sha(t["last_row"].cpu().numpy()) == ref["last_row_sha256"]
+    if "last_col_sha256" in ref and "last_col" in t:
+        ok &= sha(t["last_col"].cpu().numpy()) == ref["last_col_sha256"]
     if "image_sha256" in ref and "table" in t:
         ok &= sha(t["table"].cpu().numpy()) == ref["image_sha256"]
     return {"checked": True, "match": bool(ok), "vs": "tests/golden/bench_refs.json (oracle, seed 0)", **got}
@@ -291,53 +301,111 @@ def gather_parity(name, pb, world, rank):
     return res
 
 
+def load_latency():
+    try:
+        with open(LATENCY_FILE) as f:
+            return json.load(f)
+    except Exception:   # a-priori constants of SURVEY.md §8(d)
+        return {"lcs_cell": 4.5, "levenshtein_cell": 9.0, "dtw_cell": 10.0, "fs_cell": 28.0, "minpath_row": 11.0,
+                "_source": "a-priori (SURVEY.md 8(d))"}
+
+
 def roofline(name, ms_per_step, peaks, world, clock_mhz):
+    """the roofline time is max(T_work, T_span, T_mem); the binding term is
+    reported with its achieved / peak / frac, the others beside it."""
     cfg = CONFIGS[name]
-    cells = cfg["rows"] * cfg["cols"]
+    func, cat = cfg["func"], cfg["category"]
+    H, W = cfg["rows"], cfg["cols"]
+    cells = H * W
     t = ms_per_step / 1e3
-    if cfg["func"] == "minpath3":
-        alg_bytes = cells * 4 + cfg["cols"] * 4 + 4
-        achieved = alg_bytes / t / 1e9
-        peak = peaks.get("hbm_gbs", 6650.0) * world
-        return {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
-                "frac": round(achieved / peak, 4), "traffic": traffic_for(name),
-                "algorithmic_bytes_per_cell": 4, "peak_source": peaks.get("_source")}
-    ops = ALU_OPS_PER_CELL[cfg["func"]]
     mhz = peaks.get("sm_max_mhz", 1965.0)
-    peak = NUM_SMS * PIPE_LANES_PER_SM_CLK * mhz * 1e6 * world / 1e12
-    achieved = cells * ops / t / 1e12
-    pipe = "FMA (FP32)" if cfg["func"] in ("dtw", "fs") else "ALU (INT)"
-    return {"bound": "alu", "achieved": round(achieved, 3), "peak": round(peak, 2), "unit": "Tops/s",
-            "frac": round(achieved / peak, 4), "traffic": traffic_for(name),
-            "pipe": pipe, "algorithmic_ops_per_cell": ops,
-            "peak_derivation": f"{NUM_SMS} SMs x {PIPE_LANES_PER_SM_CLK} lanes/clk x {mhz:.0f} MHz x {world} GPU",
-            "sm_mhz_during_run": clock_mhz}
+    ops, pipe = WORK[func]
+    peak_ops = NUM_SMS * LANES[pipe] * mhz * 1e6 * world          # lane-ops / s
+    t_work = cells * ops / peak_ops
+    lat = load_latency()
+    key = {"lcs": "lcs_cell", "levenshtein": "levenshtein_cell", "dtw": "dtw_cell", "fs": "fs_cell"}.get(func, "minpath_row")
+    cyc = float(lat[key])
+    path = {"anti_diagonal": H + W - 1, "knight_move": 2 * (H - 1) + W, "prev_row": H,
+            "inverted_l": min(H, W)}[cat]                     # cells on the longest dependency path
+    t_span = path * cyc / (mhz * 1e6)
+    hbm_bytes = cells * HBM_PER_CELL.get(func, 0.0) + 4 * (H + W)
+    peak_bw = peaks.get("hbm_gbs", 6650.0) * 1e9 * world
+    t_mem = hbm_bytes / peak_bw
+    terms = {"work": t_work, "span": t_span, "mem": t_mem}
+    bound = max(terms, key=terms.get)
+    out = {"traffic": traffic_for(name), "sm_mhz_during_run": clock_mhz,
+           "terms_ms": {k: round(v * 1e3, 4) for k, v in terms.items()},
+           "frac_by_term": {k: round(v / t, 4) for k, v in terms.items()},
+           "work_per_cell": f"{ops} {'INT ALU' if pipe == 'alu' else 'FP32 FMA'} ops (SURVEY 8(d))",
+           "work_peak": f"{NUM_SMS} SMs x {LANES[pipe]} lanes/clk x {mhz:.0f} MHz x {world} GPU = {peak_ops / 1e12:.2f} T lane-ops/s",
+           "span_model": f"{path} dependent cells x {cyc:.2f} cycles ({lat.get('how', lat.get('_source', ''))})",
+           "hbm_bytes_per_step": hbm_bytes, "hbm_peak_source": peaks.get("_source")}
+    if bound == "mem":
+        ach = hbm_bytes / t / 1e9
+        out.update({"bound": "hbm", "achieved": round(ach, 1), "peak": round(peak_bw / 1e9, 1), "unit": "GB/s",
+                    "frac": round(ach / (peak_bw / 1e9), 4)})
+    elif bound == "work":
+        ach = cells * ops / t / 1e12
+        out.update({"bound": "alu" if pipe == "alu" else "fma", "achieved": round(ach, 3),
+                    "peak": round(peak_ops / 1e12, 2), "unit": "Tops/s", "frac": round(ach / (peak_ops / 1e12), 4)})
+    else:
+        ach = cells / t / 1e9
+        pk = cells / t_span / 1e9
+        out.update({"bound": "span", "achieved": round(ach, 3), "peak": round(pk, 1), "unit": "GCUPS",
+                    "frac": round(ach / pk, 4)})
+    return out
+
+
+def host_info():
+    model = ""
+    try:
+        for line in subprocess.run(["lscpu"], capture_output=True, text=True).stdout.splitlines():
+            if line.startswith("Model name:"):
+                model = line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return {"nproc": os.cpu_count(), "cpu_model": model}
 
 
 def cpu_baseline(name):
-    """The oracle as it stands, single-threaded, on a bounded sample of the workload."""
+    """The oracle as it stands, single-threaded and pinned to one core (os.sched_setaffinity, the
+    in-process equivalent of taskset -c), on a bounded sample of the workload."""
     import oracle
     cfg = CONFIGS[name]
     x = cfg["make"](0)
     func = cfg["func"]
-    t0 = time.perf_counter()
-    if func == "lcs":
-        rows = min(cfg["rows"], max(1, int(2.5e9 // cfg["cols"])))
-        oracle.lcs(x["a"][:rows], x["b"])
-        cells, sample = rows * cfg["cols"], f"first {rows} rows x all {cfg['cols']} columns"
-    elif func == "dtw":
-        rows = min(cfg["rows"], max(1, int(1.0e9 // cfg["cols"])))
-        oracle.dtw(x["a"][:rows], x["b"])
-        cells, sample = rows * cfg["cols"], f"first {rows} rows x all {cfg['cols']} columns"
-    elif func == "fs":
-        oracle.fs(x["grid"])
-        cells, sample = cfg["rows"] * cfg["cols"], "whole image"
-    else:
-        oracle.minpath3(x["grid"])
-        cells, sample = cfg["rows"] * cfg["cols"], "whole grid"
-    dt = time.perf_counter() - t0
+    try:
+        old_aff = os.sched_getaffinity(0)
+        core = min(old_aff)
+        os.sched_setaffinity(0, {core})
+    except Exception:
+        old_aff, core = None, None
+    try:
+        t0 = time.perf_counter()
+        if func == "lcs":
+            rows = min(cfg["rows"], max(1, int(2.5e9 // cfg["cols"])))
+            oracle.lcs(x["a"][:rows], x["b"])
+            cells, sample = rows * cfg["cols"], f"first {rows} rows x all {cfg['cols']} columns"
+        elif func == "dtw":
+            rows = min(cfg["rows"], max(1, int(1.0e9 // cfg["cols"])))
+            oracle.dtw(x["a"][:rows], x["b"])
+            cells, sample = rows * cfg["cols"], f"first {rows} rows x all {cfg['cols']} columns"
+        elif func == "fs":
+            oracle.fs(x["grid"])
+            cells, sample = cfg["rows"] * cfg["cols"], "whole image"
+        elif func in ("min2plus", "diagmaxplus"):
+            rows = min(cfg["rows"], 8192)
+            getattr(oracle, func)(x["grid"][:rows], cfg.get("param_c", 1))
+            cells, sample = rows * cfg["cols"], f"first {rows} rows x all {cfg['cols']} columns"
+        else:
+            oracle.minpath3(x["grid"])
+            cells, sample = cfg["rows"] * cfg["cols"], "whole grid"
+        dt = time.perf_counter() - t0
+    finally:
+        if old_aff is not None:
+            os.sched_setaffinity(0, old_aff)
     return {"value": round(cells / dt / 1e9, 4), "unit": "GCUPS", "cores": 1, "kind": "oracle",
-            "sample": sample, "seconds": round(dt, 2)}
+            "sample": sample, "seconds": round(dt, 2), "pinned_core": core, **host_info()}
 
 
 def measure(name, lddp, dev, world, rank, steps, warmup, flush, peaks, sampler, with_e2e=True,
@@ -358,6 +426,30 @@ def measure(name, lddp, dev, world, rank, steps, warmup, flush, peaks, sampler, 
                       "d2h_bytes_per_step": bo}
     if pb["comm"] is not None:
         lddp.lddp_comm_destroy(pb["comm"])
+    return out
+
+
+def scaling_model(ms1, plan, cols):
+    """column strips of n/P columns per rank.  Rank g's strip s needs rank g-1's
+    whole right column of strip s (its last chunk), so start(g, s) = s*L + g*(NQ/P + 2E) chunks
+    and the fill ends at (S-1)*L + P*(NQ/P + 2E) = T(1) + 2E(P-1) chunks: strong scaling is
+    capped at ~1x by the lane-systolic sweep (every row strip crosses all n columns one chunk at a
+    time, at the same per-chunk cost on any GPU count).  The per-chunk time t and the strip lag L
+    (2E + 1 chunks of structure + ~0.9 chunk of handoff latency, tools/l16_trace.py) are
+    calibrated on the measured N = 1 time; t_link = one NVLink store + flag hop (~2 us, assumed)."""
+    S, NQ, E = plan["strips"], plan["chunks"], plan["extra_lag"]
+    if plan.get("kernel") != "lcs16":
+        return None
+    L = 2 * E + 1.9
+    t = ms1 / (NQ + 2 * E + (S - 1) * L)
+    t_link = 2e-3
+    out = {"model": "T(P) = t*(NQ + 2E*P + (S-1)*L) + (P-1)*t_link; weak (n = cols*P): t*(P*NQ + 2E*P + (S-1)*L)",
+           "t_chunk_us": round(t * 1e3, 3), "L_chunks": L, "strips": S, "chunks": NQ}
+    for P in (1, 2, 4, 8):
+        strong = t * (NQ + 2 * E * P + (S - 1) * L) + (P - 1) * t_link
+        weak = t * (P * NQ + 2 * E * P + (S - 1) * L) + (P - 1) * t_link
+        out[f"P{P}"] = {"strong_ms": round(strong, 3), "strong_speedup": round(ms1 / strong, 3),
+                        "weak_ms": round(weak, 3), "weak_efficiency": round(ms1 / weak, 3)}
     return out
 
 
@@ -429,7 +521,7 @@ def main():
                    sampler, tile_rows=args.tile_rows)
     others = {}
     if world == 1 and not args.no_others:
-        for name in ("C1", "C2", "C3", "C4"):
+        for name in ("C1", "C2", "C3", "C4", "C6", "C7"):
             if name == args.workload:
                 continue
             r = measure(name, lddp, dev, 1, 0, max(5, args.steps // 2), args.warmup, flush, peaks, sampler,
@@ -460,6 +552,8 @@ def main():
                 "roofline": head["roofline"], "cpu_baseline": cpu, "parity": head["parity"],
                 "plan": head["plan"], "ms_min": head["ms_min"], "ms_max": head["ms_max"],
                 "configs": others}
+        if world == 1:
+            line["scaling_model"] = scaling_model(head["ms_per_step"], head["plan"], cfg["cols"])
         print(json.dumps(line), flush=True)
     if world > 1:
         import torch.distributed as dist

@@ -1,5 +1,7 @@
-"""The BASELINE.json workloads C1-C5: shapes, f, category and the
-seeded input recipe.  Shared by bench.py, tools/make_bench_refs.py and the full-size tests."""
+"""The BASELINE.json workloads C1-C5 and the two synthetic-f
+workloads of SURVEY §8(d) "(iL)" / [L298] (C6 inverted-L diagonal max-plus, C7 horizontal
+min2-plus): shapes, f, category and the seeded input recipe.  Shared by bench.py,
+tools/make_bench_refs.py and the full-size tests."""
 import os
 import sys
 
@@ -35,6 +37,12 @@ def _minpath(n):
     return make
 
 
+def _init(n):
+    def make(seed):
+        return {"grid": inputs.gen_init(seed, n, n)}
+    return make
+
+
 CONFIGS = {
     "C1": {"func": "lcs", "category": "anti_diagonal", "rows": 1024, "cols": 1024, "make": _lcs(1024),
            "desc": "LCS of two random 1024-char strings over a 4-letter alphabet (anti-diagonal, int32)"},
@@ -46,4 +54,10 @@ CONFIGS = {
            "desc": "previous-row-only 3-neighbour min-path DP on a 32768x32768 random int32 cost grid"},
     "C5": {"func": "lcs", "category": "anti_diagonal", "rows": 100000, "cols": 100000, "make": _lcs(100000),
            "desc": "LCS of two random 100000-char strings, column-strip wavefront pipeline across 1/2/4/8 B200"},
+    "C6": {"func": "diagmaxplus", "category": "inverted_l", "rows": 32768, "cols": 32768, "make": _init(32768),
+           "param_c": 1,
+           "desc": "inverted-L synthetic f = max(init, UL) + 1 [L298] on a 32768x32768 int32 grid (SURVEY 8(d) iL)"},
+    "C7": {"func": "min2plus", "category": "prev_row", "rows": 32768, "cols": 32768, "make": _init(32768),
+           "param_c": 1,
+           "desc": "horizontal case-1 synthetic f = min(UL, U) + 1 [L298] (H1) on a 32768x32768 int32 grid"},
 }
