@@ -234,14 +234,18 @@ def time_e2e(pb, lddp, steps, dev, world):
         if pb["outs"] & lddp.OUT_TABLE:
             tbl = torch.zeros((cfg["rows"], cfg["cols"]), dtype=torch.uint8).pin_memory()
             d2h = tbl.numel()
-        lr = None
+        lr = lc = None
         if pb["outs"] & lddp.OUT_LAST_ROW:
             lr = torch.zeros(cfg["cols"], dtype=cell_dt).pin_memory()
             d2h += lr.numel() * 4
-        inp, out = plan.io(a=host_in.get("a"), b=host_in.get("b"), grid=host_in.get("grid"),
-                           score=res if pb["outs"] & lddp.OUT_SCORE else None, last_row=lr, table=tbl)
-        if tbl is not None:
+        if pb["outs"] & lddp.OUT_LAST_COL:
+            lc = torch.zeros(cfg["rows"], dtype=cell_dt).pin_memory()
+            d2h += lc.numel() * 4
+        if not pb["outs"] & lddp.OUT_SCORE:
             d2h -= 4
+        inp, out = plan.io(a=host_in.get("a"), b=host_in.get("b"), grid=host_in.get("grid"),
+                           score=res if pb["outs"] & lddp.OUT_SCORE else None, last_row=lr, last_col=lc,
+                           table=tbl)
         stream = torch.cuda.current_stream(dev)
         lddp.lddp_fill_host(plan.handle, inp, out, stream.cuda_stream)   # warm staging buffers
         t0 = time.perf_counter()

@@ -6,8 +6,13 @@
 // case-1 schedule is better for coalescing [L215], [L296-L298].  On B200 the natural form is
 // neither: one lane per diagonal chain, 32 adjacent diagonals per warp, walking rows in
 // lockstep -- so lane l touches column i + d0 + l of row i: every row step is one coalesced
-// 128-byte load (and store), no inter-thread dependency at all, pure HBM streaming with an
-// unrolled prefetch of UNR rows per lane.
+// 128-byte load (and store), no inter-thread dependency at all: pure HBM streaming.
+//
+// The time of the fill is the time of the longest chains (min(H, W) rows), so each warp keeps
+// kInvlDepth rows of loads in flight (two register blocks: the next block is loaded while the
+// current one is evaluated): 2048 warps x 64 rows x 128 B = 16 MB in flight for C6, enough to
+// cover the HBM latency at full bandwidth.  Every warp owns one group of 32
+// diagonals for the whole fill (the grid holds all of them: no tail of late-starting chains).
 #include <cstdint>
 #include "cellfn.cuh"
 #include "params.h"
@@ -15,8 +20,8 @@
 
 namespace lddp {
 
-constexpr int kInvlWarps = 8;
-constexpr int kInvlUnroll = 8;
+constexpr int kInvlWarps = 4;
+constexpr int kInvlBlock = 32;   // rows per register block (two blocks in flight)
 
 template <class F, bool TABLE>
 __global__ void __launch_bounds__(kInvlWarps * 32) invl_kernel(const FillParams p) {
@@ -38,28 +43,37 @@ __global__ void __launch_bounds__(kInvlWarps * 32) invl_kernel(const FillParams 
     const int64_t dhi = min((int64_t)W - 1, dlo + 31);
     const int64_t ibeg = max((int64_t)0, -dhi);
     const int64_t iend = min(H, (int64_t)W - dlo);   // exclusive
+    // this lane's chain: rows [ia, ib)
+    const int64_t ia = max((int64_t)0, -d), ib = min(H, (int64_t)W - d);
+    const G* src = static_cast<const G*>(p.grid) + d;   // element (i, i + d) = src + i * (pitch + 1)
+    const int64_t step = p.grid_pitch + 1;
     T v = T(0);
-    for (int64_t i0 = ibeg; i0 < iend; i0 += kInvlUnroll) {
-      G g[kInvlUnroll];
+    G cur[kInvlBlock], nxt[kInvlBlock];
+    auto load_block = [&](G* dst, int64_t i0) {
 #pragma unroll
-      for (int u = 0; u < kInvlUnroll; ++u) {
+      for (int u = 0; u < kInvlBlock; ++u) {
         const int64_t i = i0 + u;
-        const int64_t j = i + d;
-        g[u] = (live && i < iend && j >= 0 && j < W) ? F::load(p, i, (int)j) : G(0);
+        dst[u] = (live && i >= ia && i < ib) ? __ldcs(src + i * step) : G(0);
       }
+    };
+    load_block(cur, ibeg);
+    for (int64_t i0 = ibeg; i0 < iend; i0 += kInvlBlock) {
+      if (i0 + kInvlBlock < iend) load_block(nxt, i0 + kInvlBlock);
 #pragma unroll
-      for (int u = 0; u < kInvlUnroll; ++u) {
+      for (int u = 0; u < kInvlBlock; ++u) {
         const int64_t i = i0 + u;
         const int64_t j = i + d;
-        if (live && i < iend && j >= 0 && j < W) {
+        if (live && i >= ia && i < ib) {
           typename F::OutT o;
-          v = F::f(v, v, v, v, typename F::RowCtx(0), typename F::ColCtx(0), g[u], i,
+          v = F::f(v, v, v, v, typename F::RowCtx(0), typename F::ColCtx(0), cur[u], i,
                    (int)j + p.col0, p.param_c, o);
           if (TABLE) static_cast<typename F::OutT*>(p.table)[i * p.table_pitch + j] = o;
           if (i == H - 1 && p.last_row != nullptr) static_cast<T*>(p.last_row)[j] = v;
           if (j == W - 1 && p.last_col != nullptr) static_cast<T*>(p.last_col)[i] = v;
         }
       }
+#pragma unroll
+      for (int u = 0; u < kInvlBlock; ++u) cur[u] = nxt[u];
     }
   }
 }

@@ -180,7 +180,7 @@ constexpr int kPrevBandRows = 64;     // must match prevrow.cu
 constexpr int kPrevBW = 128;
 constexpr int kPrevRing = 4;
 constexpr int kPrevThreads = 256;
-constexpr int kInvlThreads = 256;
+constexpr int kInvlThreads = 128;   // must match invl.cu (kInvlWarps x 32)
 
 int env_int(const char* name, int dflt) {
   const char* v = getenv(name);
@@ -698,7 +698,7 @@ lddp_status lddp_plan(const lddp_desc* desc, lddp_plan_t* out) {
       const int64_t nd = d.rows + d.cols - 1;
       const int64_t warps = (nd + 31) / 32;
       const int64_t blocks = (warps + (kInvlThreads / 32) - 1) / (kInvlThreads / 32);
-      pl->grid = (int)std::max<int64_t>(1, std::min<int64_t>(blocks, (int64_t)pl->sms * 8));
+      pl->grid = (int)std::max<int64_t>(1, std::min<int64_t>(blocks, (int64_t)pl->sms * 16));   // every diagonal group resident
       pl->off_prog = 64;
       pl->off_bnd = 64;
       pl->ws_bytes = 64;
