@@ -58,6 +58,10 @@ def _L():
         lib.oracle_min2plus.argtypes = [p, i64, i64, ctypes.c_int32, p, i64, p]
         lib.oracle_diagmaxplus.restype = None
         lib.oracle_diagmaxplus.argtypes = [p, i64, i64, ctypes.c_int32, p, i64, p, p]
+        lib.oracle_min2plus_v.restype = ctypes.c_int32
+        lib.oracle_min2plus_v.argtypes = [p, i64, i64, ctypes.c_int32, p, i64, p]
+        lib.oracle_antidiag_maxplus.restype = None
+        lib.oracle_antidiag_maxplus.argtypes = [p, i64, i64, ctypes.c_int32, p, i64, p, p]
         _lib = lib
     return _lib
 
@@ -147,6 +151,29 @@ def min2plus(init, c: int = 1, table: bool = False) -> Result:
 def diagmaxplus(init, c: int = 1, table: bool = False) -> Result:
     """Inverted-L synthetic f = max(init, UL) + c ([L298] §V.B)."""
     return _grid_fill(_L().oracle_diagmaxplus, init, (int(c),), table, want_col=True)
+
+
+def min2plus_v(init, c: int = 1, table: bool = False) -> Result:
+    """Vertical twin of min2plus ([L111], reading R15): f = min(L, UL) + c, column 0 = init.
+    Returns score = min of the last column, last_col, table."""
+    grid = _c(init, np.int32)
+    H, W = grid.shape
+    tab = np.empty((H, W), np.int32) if table else None
+    last_col = np.empty(H, np.int32)
+    score = _L().oracle_min2plus_v(_ptr(grid), H, W, int(c), _ptr(tab), W, _ptr(last_col))
+    return Result(score=score, last_col=last_col, table=tab)
+
+
+def antidiag_maxplus(init, c: int = 1, table: bool = False) -> Result:
+    """mInverted-L twin of diagmaxplus ([L111], reading R15): f = max(init, UR) + c, row 0 and
+    column W-1 = init.  Returns last_row and last_col = COLUMN 0 (where its chains end), table."""
+    grid = _c(init, np.int32)
+    H, W = grid.shape
+    tab = np.empty((H, W), np.int32) if table else None
+    last_row = np.empty(W, np.int32)
+    first_col = np.empty(H, np.int32)
+    _L().oracle_antidiag_maxplus(_ptr(grid), H, W, int(c), _ptr(tab), W, _ptr(last_row), _ptr(first_col))
+    return Result(last_row=last_row, last_col=first_col, table=tab)
 
 
 def traceback(func: str, a, b, table):

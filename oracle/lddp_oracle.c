@@ -299,3 +299,67 @@ void oracle_diagmaxplus(const int32_t* init, int64_t H, int64_t W, int32_t cst,
     if (last_row) memcpy(last_row, prev, (size_t)W * sizeof(int32_t));
     free(prev); free(cur);
 }
+
+/* ------------------------------------------------------------------------------------------
+ * The two symmetric twins of Table I [L109-L113] ("Vertical is the transpose of Horizontal,
+ * mInverted-L the mirror of Inverted-L" [L111]), instantiated with the synthetic f's of §V.B
+ * [L298] so that every one of the six patterns has a compiled-in f (reading R15).
+ *
+ * MIN2_PLUS_V (Vertical, contributing set {L, UL}, Table I [L137]):
+ *   f(i,0) = init[i][0] (column 0 is the boundary);  f(0,j) = f(0,j-1) + c (only L exists);
+ *   f(i,j) = min(f(i,j-1), f(i-1,j-1)) + c.
+ * Outputs: last_col (the right column, where the column sweep ends) and its minimum.
+ * ---------------------------------------------------------------------------------------- */
+int32_t oracle_min2plus_v(const int32_t* init, int64_t H, int64_t W, int32_t cst,
+                          int32_t* table, int64_t pitch, int32_t* last_col)
+{
+    if (H <= 0 || W <= 0) return 0;
+    int32_t* prev = (int32_t*)malloc((size_t)W * sizeof(int32_t));
+    int32_t* cur  = (int32_t*)malloc((size_t)W * sizeof(int32_t));
+    int32_t best = 0;
+    for (int64_t i = 0; i < H; ++i) {
+        for (int64_t j = 0; j < W; ++j) {
+            if (j == 0) {
+                cur[j] = init[i * W];
+            } else {
+                int32_t m = cur[j - 1];                           /* L  */
+                if (i > 0 && prev[j - 1] < m) m = prev[j - 1];    /* UL */
+                cur[j] = m + cst;
+            }
+        }
+        if (table) memcpy(table + i * pitch, cur, (size_t)W * sizeof(int32_t));
+        if (last_col) last_col[i] = cur[W - 1];
+        if (i == 0 || cur[W - 1] < best) best = cur[W - 1];
+        int32_t* t = prev; prev = cur; cur = t;
+    }
+    free(prev); free(cur);
+    return best;
+}
+
+/* ANTIDIAG_MAXPLUS (mInverted-L, contributing set {UR}, Table I [L126]):
+ *   f(i,j) = init[i][j] on row 0 and on column W-1 (the boundary);
+ *   f(i,j) = max(init[i][j], f(i-1,j+1)) + c.
+ * Its chains run down-left and end on the last row or on column 0.  Outputs: last_row and
+ * first_col (column 0, where the chains end). */
+void oracle_antidiag_maxplus(const int32_t* init, int64_t H, int64_t W, int32_t cst,
+                             int32_t* table, int64_t pitch, int32_t* last_row, int32_t* first_col)
+{
+    if (H <= 0 || W <= 0) return;
+    int32_t* prev = (int32_t*)malloc((size_t)W * sizeof(int32_t));
+    int32_t* cur  = (int32_t*)malloc((size_t)W * sizeof(int32_t));
+    for (int64_t i = 0; i < H; ++i) {
+        for (int64_t j = 0; j < W; ++j) {
+            int32_t v = init[i * W + j];
+            if (i > 0 && j < W - 1) {
+                if (prev[j + 1] > v) v = prev[j + 1];             /* UR */
+                v += cst;
+            }
+            cur[j] = v;
+        }
+        if (table) memcpy(table + i * pitch, cur, (size_t)W * sizeof(int32_t));
+        if (first_col) first_col[i] = cur[0];
+        int32_t* t = prev; prev = cur; cur = t;
+    }
+    if (last_row) memcpy(last_row, prev, (size_t)W * sizeof(int32_t));
+    free(prev); free(cur);
+}

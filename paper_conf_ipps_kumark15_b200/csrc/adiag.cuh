@@ -143,8 +143,8 @@ struct AdWarp {
   uint64_t tp;      // this lane's top pair of the current chunk (column 32k + lane)
   uint64_t tq1;     // global top prefetch (chunk k+1)
   const uint64_t* tqsrc;   // TS 2: this lane's slot of the previous strip's boundary row (column
-                           // 32k + lane at tqsrc + 32k); the next chunk's pair is loaded half a
-                           // chunk ahead (at group 2), late enough to be published already
+                           // 32k + lane at tqsrc + 32k); the next chunk's pair is loaded inside the
+                           // group loop at group kAdPfGroup (0 for LCS / Levenshtein, 2 for DTW)
   int tqn;                 // chunks with a global top pair (NQ), 0 for other roles
   long long wait_top; // clock64 cycles spent waiting for top values (trace builds)
 

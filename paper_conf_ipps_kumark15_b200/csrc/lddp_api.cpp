@@ -565,9 +565,10 @@ lddp_status lddp_plan(const lddp_desc* desc, lddp_plan_t* out) {
       // DTW: one warp per strip (every handoff through the global boundary rows, prefetched half
       // a chunk ahead) measured best on B200 (C2 0.93 -> 0.85 ms against 4-warp CTAs)
       if (Wq <= 0 && d.func == LDDP_F_DTW) Wq = 1;
-      // LCS / Levenshtein: one warp per strip too when the strips of 192 rows fit one wave of
-      // CTAs (small tables, C1 0.084 -> 0.080 ms); 4-warp CTAs with shared rings otherwise
-      // (C5: 521 one-warp strips measured 8.2 ms against 6.6)
+      // Levenshtein (and LCS with LDDP_KERNEL=adiag): one-warp strips as well -- every handoff
+      // through the global boundary rows, the next chunk's pairs prefetched inside the group loop
+      // (measured best for C5 in round 1: 5.80 ms against 6.58 with 4-warp CTAs and shared rings);
+      // with W = 1 forced, the cost model below only chooses among the W = 1 geometries
       if (Wq <= 0 && d.func != LDDP_F_DTW) {
         for (const auto& g : kAdGeoms)
           if (g.func == d.func && g.W == 1) { Wq = 1; break; }
@@ -580,7 +581,6 @@ lddp_status lddp_plan(const lddp_desc* desc, lddp_plan_t* out) {
         if (Wq > 0 && g.W != Wq) continue;
         if (Sq >= 0 && g.S != Sq) continue;
         if (Sq < 0 && g.S) continue;   // split geometries only on request: measured slower on B200 (C5 6.9 -> 11.6 ms)
-        if (Wq <= 0 && g.W < 4) continue;   // 1-2 warp CTAs only on request: measured slower (C5 7.3-8.2 ms)
         double c = ad_cost(d.func, g.R, g.E, g.W, g.S, d.rows, std::max<int64_t>(d.cols, 1), pl->sms);
         if (Rq > 0) c += 1e200 * std::abs(g.R - Rq);   // nearest compiled R to the request
         if (getenv("LDDP_PLAN_DEBUG"))
@@ -797,16 +797,21 @@ lddp_status lddp_fill_host(lddp_plan_t pl, const lddp_inputs* hin, const lddp_ou
     cudaStream_t s = (cudaStream_t)stream;
     const lddp_desc& d = pl->desc;
     std::lock_guard<std::mutex> lk(pl->mu);
+    // device staging rows are re-pitched to 16-byte multiples whatever the host pitch (the FS /
+    // prev-row fast paths need 16-byte aligned rows; the host pitch never reaches a kernel)
+    const size_t gel = grid_elt_bytes(d.func), tel = table_elt_bytes(d.func);
+    const size_t gdp = align_up((size_t)std::max<int64_t>(d.cols, 1) * gel, 16);
+    const size_t tdp = align_up((size_t)std::max<int64_t>(d.cols, 1) * tel, 16);
     size_t need[6] = {0, 0, 0, 0, 0, 0};
     if (seq_func(d.func)) {
       need[0] = d.rows * seq_elt_bytes(d.func);
       need[1] = d.cols * seq_elt_bytes(d.func);
     } else {
-      need[2] = d.rows * hin->grid_pitch * grid_elt_bytes(d.func);
+      need[2] = d.rows * gdp;
     }
     need[3] = (d.outputs & LDDP_OUT_LAST_ROW) ? d.cols * cell_bytes(d.func) : 0;
     need[4] = (d.outputs & LDDP_OUT_LAST_COL) ? d.rows * cell_bytes(d.func) : 0;
-    need[5] = (d.outputs & LDDP_OUT_TABLE) ? d.rows * hout->table_pitch * table_elt_bytes(d.func) + 16 : 16;
+    need[5] = (d.outputs & LDDP_OUT_TABLE) ? d.rows * tdp + 16 : 16;
     for (int k = 0; k < 6; ++k) {
       if (need[k] > pl->stage_bytes[k]) {
         if (pl->stage[k]) cudaFree(pl->stage[k]);
@@ -820,7 +825,13 @@ lddp_status lddp_fill_host(lddp_plan_t pl, const lddp_inputs* hin, const lddp_ou
     lddp_outputs dout = *hout;
     if (need[0]) { CUDA_TRY(cudaMemcpyAsync(pl->stage[0], hin->a, need[0], cudaMemcpyHostToDevice, s)); din.a = pl->stage[0]; }
     if (need[1]) { CUDA_TRY(cudaMemcpyAsync(pl->stage[1], hin->b, need[1], cudaMemcpyHostToDevice, s)); din.b = pl->stage[1]; }
-    if (need[2]) { CUDA_TRY(cudaMemcpyAsync(pl->stage[2], hin->grid, need[2], cudaMemcpyHostToDevice, s)); din.grid = pl->stage[2]; }
+    if (need[2]) {
+      CUDA_TRY(cudaMemcpy2DAsync(pl->stage[2], gdp, hin->grid, hin->grid_pitch * gel, d.cols * gel, d.rows,
+                                 cudaMemcpyHostToDevice, s));
+      din.grid = pl->stage[2];
+      din.grid_pitch = (int64_t)(gdp / gel);
+    }
+    if (d.outputs & LDDP_OUT_TABLE) dout.table_pitch = (int64_t)(tdp / tel);
     char* score_dev = static_cast<char*>(pl->stage[5]) + ((d.outputs & LDDP_OUT_TABLE) ? need[5] - 16 : 0);
     dout.score = hout->score ? score_dev : nullptr;
     dout.last_row = need[3] ? pl->stage[3] : nullptr;
@@ -841,8 +852,9 @@ lddp_status lddp_fill_host(lddp_plan_t pl, const lddp_inputs* hin, const lddp_ou
       CUDA_TRY(cudaMemcpyAsync(hout->score, score_dev, cell_bytes(d.func), cudaMemcpyDeviceToHost, s));
     if (need[3]) CUDA_TRY(cudaMemcpyAsync(hout->last_row, pl->stage[3], need[3], cudaMemcpyDeviceToHost, s));
     if (need[4]) CUDA_TRY(cudaMemcpyAsync(hout->last_col, pl->stage[4], need[4], cudaMemcpyDeviceToHost, s));
-    if (d.outputs & LDDP_OUT_TABLE)
-      CUDA_TRY(cudaMemcpyAsync(hout->table, pl->stage[5], need[5] - 16, cudaMemcpyDeviceToHost, s));
+    if ((d.outputs & LDDP_OUT_TABLE) && d.rows > 0 && d.cols > 0)
+      CUDA_TRY(cudaMemcpy2DAsync(hout->table, hout->table_pitch * tel, pl->stage[5], tdp, d.cols * tel, d.rows,
+                                 cudaMemcpyDeviceToHost, s));
     CUDA_TRY(cudaStreamSynchronize(s));
     return lddp_status_check(pl, ws, stream);
   } catch (...) {

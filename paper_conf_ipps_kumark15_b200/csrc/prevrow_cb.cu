@@ -16,7 +16,7 @@
 //    published edges: case-2 two-way halo of Table II [L265-L274], ([L193-L195]), one exchange
 //    per HB rows instead of one per row.
 //  * Edge exchange = (value, tag) 64-bit pairs in global memory (single-copy atomic): the
-//    consumer polls the data itself, no flag, no fence.  Tag = hash(fill epoch) + band.
+//    consumer polls the data itself, no flag, no fence.  Tag = (fill epoch mod 4096) << 20 | band + 1.
 //  * Cost rows (the HBM stream, 4 B/cell) flow through a per-warp D-row shared-memory ring
 //    filled by 16-byte cp.async (LDGSTS.128, L1 bypass; 8-byte when VP % 4 != 0), D-1 rows ahead
 //    of the row being computed; every lane copies exactly the columns it later reads, so the ring
@@ -344,7 +344,9 @@ __global__ void __launch_bounds__(256) prevrow_cb_kernel(const FillParams p, con
 #pragma unroll
     for (int v = 0; v < VP; ++v) cur[v] = ((omask >> v) & 1u) ? outv[v] : F::top(p, e0 + v);
 
-    const uint32_t tag0 = (uint32_t)(p.epoch * 0x9E3779B1ull);
+    // edge-pair tags: fill epoch (mod 4096) and band + 1 in disjoint bit fields -- every slot a fill
+  // uses is rewritten by it, so a pair left by an earlier fill of this workspace never matches
+  const uint32_t tag0 = (uint32_t)(p.epoch & 0xFFFu) << 20;
     uint64_t* edges = reinterpret_cast<uint64_t*>(p.bnd);   // [nb][4 slots][2 sides][HB] pairs
     const bool lhalo = lane < HL, rhalo = lane >= 32 - HL;
     const bool ledge = lane >= HL && lane < 2 * HL;          // own columns [j0, j0 + HB)
@@ -367,7 +369,7 @@ __global__ void __launch_bounds__(256) prevrow_cb_kernel(const FillParams p, con
       if (p.debug & 8) continue;   // development: no band exchange (wrong results; timing only)
       // ---- band boundary: publish own edges, take the neighbours' as halos
       const int band = (int)(r0 / HB);
-      const uint32_t tag = tag0 + (uint32_t)band + 1u;
+      const uint32_t tag = tag0 | (((uint32_t)band + 1u) & 0xFFFFFu);
       uint64_t* mine = edges + ((size_t)q * 4 + (band & 3)) * 2 * HB;
       if (ledge || redge) {
         uint64_t* d = mine + (ledge ? 0 : HB) + (ledge ? (lane - HL) : (lane - (32 - 2 * HL))) * VP;
@@ -547,7 +549,9 @@ __global__ void __launch_bounds__(256) prevrow_gh_kernel(const FillParams p, con
     }
   };
 
-  const uint32_t tag0 = (uint32_t)(p.epoch * 0x9E3779B1ull);
+  // edge-pair tags: fill epoch (mod 4096) and band + 1 in disjoint bit fields -- every slot a fill
+  // uses is rewritten by it, so a pair left by an earlier fill of this workspace never matches
+  const uint32_t tag0 = (uint32_t)(p.epoch & 0xFFFu) << 20;
   uint64_t* edges = reinterpret_cast<uint64_t*>(p.bnd);
   const bool lhalo = lane < HL, rhalo = lane >= 32 - HL;
   const bool ledge = lane >= HL && lane < 2 * HL;
@@ -602,7 +606,7 @@ __global__ void __launch_bounds__(256) prevrow_gh_kernel(const FillParams p, con
     else band(nr, r0, std::false_type{});
     if (r0 + HB >= H) break;
     const int bnd_ = (int)(r0 / HB);
-    const uint32_t tag = tag0 + (uint32_t)bnd_ + 1u;
+    const uint32_t tag = tag0 | (((uint32_t)bnd_ + 1u) & 0xFFFFFu);
     uint64_t* mine = edges + ((size_t)q * 4 + (bnd_ & 3)) * 2 * HB;
     if (ledge || redge) {
       uint64_t* d = mine + (ledge ? 0 : HB) + (ledge ? (lane - HL) : (lane - (32 - 2 * HL))) * VP;

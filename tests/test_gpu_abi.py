@@ -18,7 +18,7 @@ def L():
 
 
 def _host_fill(L, func, category, outputs, a=None, b=None, grid=None, table_shape=None,
-               cell=np.int32):
+               cell=np.int32, table_pitch=None):
     rows, cols = (len(a), len(b)) if grid is None else grid.shape
     d = L.lddp_desc(rows=rows, cols=cols, category=L.CATEGORIES[category], func=L.FUNCS[func],
                     outputs=outputs, param_c=1)
@@ -27,12 +27,13 @@ def _host_fill(L, func, category, outputs, a=None, b=None, grid=None, table_shap
         score = np.full(1, -7, cell)
         last_row = np.full(max(cols, 1), -7, cell)
         last_col = np.full(max(rows, 1), -7, cell)
-        table = None if table_shape is None else np.zeros(table_shape, np.uint8)
+        tbl_full = None if table_shape is None else np.zeros((table_shape[0], table_pitch or table_shape[1]), np.uint8)
+        table = None if tbl_full is None else tbl_full[:, :table_shape[1]]
         ptr = lambda x: None if x is None else x.ctypes.data
         inp = L.lddp_inputs(a=ptr(a), b=ptr(b), grid=ptr(grid),
                             grid_pitch=0 if grid is None else grid.strides[0] // grid.itemsize)
         out = L.lddp_outputs(score=ptr(score), last_row=ptr(last_row), last_col=ptr(last_col),
-                             table=ptr(table), table_pitch=0 if table is None else table.shape[1])
+                             table=ptr(tbl_full), table_pitch=0 if table is None else tbl_full.shape[1])
         for _ in range(3):   # repeated calls reuse the plan's staging buffers and workspace
             L.lddp_fill_host(plan, inp, out, 0)
         return score[0], last_row[:cols], last_col[:rows], table
@@ -60,6 +61,23 @@ def test_fill_host_fs_and_minpath(L):
     np.testing.assert_array_equal(out, oracle.fs(img))
     c = inputs.gen_costs(4, 300, 500)
     ref = oracle.minpath3(c)
+    s, lr, _, _ = _host_fill(L, "minpath3", "prev_row", L.OUT_SCORE | L.OUT_LAST_ROW, grid=c)
+    assert s == ref.score
+    np.testing.assert_array_equal(lr, ref.last_row)
+
+
+@pytest.mark.parametrize("H,W,gpitch,tpitch", [(300, 401, 401, 401), (257, 333, 340, 335), (100, 64, 71, 64),
+                                                 (129, 96, 96, 99)])
+def test_fill_host_fs_odd_pitches(L, H, W, gpitch, tpitch):
+    """Host images and output tables with any pitch (odd widths, pitches not multiples of 4 or 16):
+    lddp_fill_host re-pitches its device staging rows, so the word-wide / 16-byte FS paths never
+    see a misaligned row."""
+    full = inputs.gen_image(H + W, H, gpitch, "uniform")
+    img = full[:, :W]
+    *_, out = _host_fill(L, "fs", "knight_move", L.OUT_TABLE, grid=img, table_shape=(H, W), table_pitch=tpitch)
+    np.testing.assert_array_equal(out, oracle.fs(np.ascontiguousarray(img)))
+    c = inputs.gen_costs(H, H, gpitch)[:, :W]
+    ref = oracle.minpath3(np.ascontiguousarray(c))
     s, lr, _, _ = _host_fill(L, "minpath3", "prev_row", L.OUT_SCORE | L.OUT_LAST_ROW, grid=c)
     assert s == ref.score
     np.testing.assert_array_equal(lr, ref.last_row)

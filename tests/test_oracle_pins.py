@@ -409,6 +409,77 @@ def test_diagmaxplus_constant(oracle_mod):
     assert np.all(r.table == 5)
 
 
+# ------------------------------------------------- symmetric twins (Vertical, mInverted-L)
+
+
+def test_min2plus_v_closed_form(oracle_mod):
+    """Vertical twin: f(i,j) = j*c + min(init[max(0, i-j) .. i][0]) -- a sliding-window min of
+    column 0 (the transpose of min2plus's closed form)."""
+    rng = np.random.default_rng(29)
+    for _ in range(30):
+        H, W = int(rng.integers(1, 40)), int(rng.integers(1, 40))
+        cst = int(rng.integers(0, 5))
+        init = inputs.gen_init(int(rng.integers(1 << 30)), H, W, hi=1000)
+        r = oracle_mod.min2plus_v(init, cst, table=True)
+        for j in range(W):
+            ref = [j * cst + init[max(0, i - j): i + 1, 0].min() for i in range(H)]
+            np.testing.assert_array_equal(r.table[:, j], ref)
+        np.testing.assert_array_equal(r.last_col, r.table[:, -1])
+        assert r.score == r.table[:, -1].min()
+
+
+def test_min2plus_v_brute_paths(oracle_mod):
+    """f(i,j) = min over monotone paths of right / up-right moves from column 0 to (i, j)."""
+    init = inputs.gen_init(3, 6, 5, hi=100)
+    cst = 2
+    r = oracle_mod.min2plus_v(init, cst, table=True)
+    H, W = init.shape
+    for i in range(H):
+        for j in range(W):
+            best = None
+            for moves in itertools.product((0, 1), repeat=j):    # right (L) or down-right (UL)
+                i0 = i - sum(moves)
+                if i0 >= 0:
+                    v = int(init[i0, 0]) + j * cst
+                    best = v if best is None else min(best, v)
+            assert r.table[i, j] == best
+
+
+def test_antidiag_maxplus_closed_form(oracle_mod):
+    """mInverted-L twin: along each anti-diagonal chain (i-k, j+k) the recurrence unrolls into an
+    offset prefix-max: f(i,j) = max(max_{k<K} init[i-k][j+k] + (k+1)c, init[i-K][j+K] + K c),
+    K = min(i, W-1-j)."""
+    rng = np.random.default_rng(31)
+    for _ in range(30):
+        H, W = int(rng.integers(1, 30)), int(rng.integers(1, 30))
+        cst = int(rng.integers(0, 4))
+        init = inputs.gen_init(int(rng.integers(1 << 30)), H, W, hi=50)
+        r = oracle_mod.antidiag_maxplus(init, cst, table=True)
+        for i in range(H):
+            for j in range(W):
+                K = min(i, W - 1 - j)
+                cands = [int(init[i - k, j + k]) + (k + 1) * cst for k in range(K)]
+                cands.append(int(init[i - K, j + K]) + K * cst)
+                assert r.table[i, j] == max(cands)
+        np.testing.assert_array_equal(r.last_row, r.table[-1])
+        np.testing.assert_array_equal(r.last_col, r.table[:, 0])
+
+
+def test_twins_are_transpose_and_mirror(oracle_mod):
+    """[L111]: Vertical = transpose of Horizontal, mInverted-L = mirror of Inverted-L.  The twin
+    oracles equal the transposed / mirrored runs of the (separately pinned) originals."""
+    rng = np.random.default_rng(37)
+    for _ in range(10):
+        H, W = int(rng.integers(1, 50)), int(rng.integers(1, 50))
+        init = inputs.gen_init(int(rng.integers(1 << 30)), H, W, hi=1 << 20)
+        v = oracle_mod.min2plus_v(init, 3, table=True)
+        h = oracle_mod.min2plus(np.ascontiguousarray(init.T), 3, table=True)
+        np.testing.assert_array_equal(v.table, h.table.T)
+        a = oracle_mod.antidiag_maxplus(init, 2, table=True)
+        d = oracle_mod.diagmaxplus(np.ascontiguousarray(init[:, ::-1]), 2, table=True)
+        np.testing.assert_array_equal(a.table, d.table[:, ::-1])
+
+
 # -------------------------------------------------------------------- Table I / Fig. 2
 
 
