@@ -63,7 +63,13 @@ typedef enum {
     LDDP_CAT_PREV_ROW = 0,      /* "Horizontal" [L180-L195]: t = i.  Masks within {UL,U,UR}      */
     LDDP_CAT_ANTI_DIAGONAL = 1, /* [L148-L168]: t = i + j.  Masks within {L,UL,U}                */
     LDDP_CAT_KNIGHT_MOVE = 2,   /* "all-four-neighbour skewed" [L217-L241]: t = 2i + j.  Any mask */
-    LDDP_CAT_INVERTED_L = 3     /* the remaining pattern [L197-L215]: t = min(i,j).  Mask {UL}   */
+    LDDP_CAT_INVERTED_L = 3,    /* the remaining pattern [L197-L215]: t = min(i,j).  Mask {UL}   */
+    /* The two symmetric twins of Table I [L109-L113]: "Vertical is the transpose of Horizontal,
+     * mInverted-L the mirror of Inverted-L" [L111].  They run on the kernels of their twins. */
+    LDDP_CAT_VERTICAL = 4,      /* t = j (column sweep).  Mask within {L,UL}.  Transpose (a tiled
+                                   transpose kernel into the workspace) + the prev-row kernel   */
+    LDDP_CAT_MINVERTED_L = 5    /* t = min(i, W-1-j).  Mask {UR}.  The inverted-L kernel reading
+                                   the grid mirrored (column j <-> W-1-j), no copy              */
 } lddp_category;
 
 /* The six patterns of Table I (lddp_classify reports the paper's pattern for a mask). */
@@ -95,7 +101,13 @@ typedef enum {
  *  DIAG_MAXPLUS [L298] f = max(init[i][j], f(i-1,j-1)) + c; row 0 / col 0 = init.  {UL}.
  *  MIN2_PLUS    [L298] f = min(f(i-1,j-1), f(i-1,j)) + c; row 0 = init; j=0 uses U only. {UL,U}.
  *  LEVENSHTEIN  [L319-L329] f = max(i,j) if min(i,j)=0; UL if a_i=b_j; else 1+min(U,L,UL).
- *               Same layout as LCS.  mask {L,UL,U}.                                            */
+ *               Same layout as LCS.  mask {L,UL,U}.
+ *  MIN2_PLUS_V  the Vertical twin of MIN2_PLUS (reading R15): f = min(L, UL) + c; column 0 =
+ *               init; row 0 uses L only.  SCORE = min of the last column.  mask {L,UL};
+ *               category VERTICAL only.
+ *  ANTIDIAG_MAXPLUS  the mInverted-L twin of DIAG_MAXPLUS (R15): f = max(init, UR) + c; row 0
+ *               and column W-1 = init.  LAST_COL = column 0 (where its chains end).  mask {UR};
+ *               category MINVERTED_L only.                                                      */
 typedef enum {
     LDDP_F_LCS = 0,
     LDDP_F_DTW = 1,
@@ -103,7 +115,9 @@ typedef enum {
     LDDP_F_MIN_PATH3 = 3,
     LDDP_F_DIAG_MAXPLUS = 4,
     LDDP_F_MIN2_PLUS = 5,
-    LDDP_F_LEVENSHTEIN = 6
+    LDDP_F_LEVENSHTEIN = 6,
+    LDDP_F_MIN2_PLUS_V = 7,
+    LDDP_F_ANTIDIAG_MAXPLUS = 8
 } lddp_func;
 
 /* Requested outputs (bitmask). */
@@ -111,7 +125,8 @@ typedef enum {
                                  int32 min of the last row.  Not valid for FS / DIAG_MAXPLUS.   */
 #define LDDP_OUT_LAST_ROW 2u  /* bottom row of the region: cols elements                        */
 #define LDDP_OUT_LAST_COL 4u  /* right column of the region: rows elements (anti-diagonal,
-                                 knight-move and inverted-L categories)                          */
+                                 knight-move, inverted-L and vertical categories; column 0 for
+                                 ANTIDIAG_MAXPLUS).  Not produced by the prev-row category.      */
 #define LDDP_OUT_TABLE    8u  /* whole region, row-major, pitch outputs.table_pitch elements.
                                  Always required (and implied) for FS_DITHER (output image).    */
 

@@ -23,7 +23,8 @@ namespace lddp {
 constexpr int kInvlWarps = 4;
 constexpr int kInvlBlock = 32;   // rows per register block (two blocks in flight)
 
-template <class F, bool TABLE>
+// MIRROR: the kernel's column j' is the grid's column W-1-j' (mInverted-L twin, {UR} -> {UL}).
+template <class F, bool TABLE, bool MIRROR>
 __global__ void __launch_bounds__(kInvlWarps * 32) invl_kernel(const FillParams p) {
   using T = typename F::T;
   using G = typename F::GridT;
@@ -45,8 +46,9 @@ __global__ void __launch_bounds__(kInvlWarps * 32) invl_kernel(const FillParams 
     const int64_t iend = min(H, (int64_t)W - dlo);   // exclusive
     // this lane's chain: rows [ia, ib)
     const int64_t ia = max((int64_t)0, -d), ib = min(H, (int64_t)W - d);
-    const G* src = static_cast<const G*>(p.grid) + d;   // element (i, i + d) = src + i * (pitch + 1)
-    const int64_t step = p.grid_pitch + 1;
+    // element (i, i + d) = src + i * step (mirrored: grid column W-1-(i+d))
+    const G* src = static_cast<const G*>(p.grid) + (MIRROR ? (int64_t)W - 1 - d : d);
+    const int64_t step = MIRROR ? p.grid_pitch - 1 : p.grid_pitch + 1;
     T v = T(0);
     G cur[kInvlBlock], nxt[kInvlBlock];
     auto load_block = [&](G* dst, int64_t i0) {
@@ -67,8 +69,9 @@ __global__ void __launch_bounds__(kInvlWarps * 32) invl_kernel(const FillParams 
           typename F::OutT o;
           v = F::f(v, v, v, v, typename F::RowCtx(0), typename F::ColCtx(0), cur[u], i,
                    (int)j + p.col0, p.param_c, o);
-          if (TABLE) static_cast<typename F::OutT*>(p.table)[i * p.table_pitch + j] = o;
-          if (i == H - 1 && p.last_row != nullptr) static_cast<T*>(p.last_row)[j] = v;
+          const int64_t jg = MIRROR ? (int64_t)W - 1 - j : j;   // the grid's column
+          if (TABLE) static_cast<typename F::OutT*>(p.table)[i * p.table_pitch + jg] = o;
+          if (i == H - 1 && p.last_row != nullptr) static_cast<T*>(p.last_row)[jg] = v;
           if (j == W - 1 && p.last_col != nullptr) static_cast<T*>(p.last_col)[i] = v;
         }
       }
@@ -78,20 +81,20 @@ __global__ void __launch_bounds__(kInvlWarps * 32) invl_kernel(const FillParams 
   }
 }
 
-template <class F>
+template <class F, bool MIRROR>
 static cudaError_t launch_il(const FillParams& p, int grid, cudaStream_t s) {
   if (p.table != nullptr)
-    invl_kernel<F, true><<<grid, kInvlWarps * 32, 0, s>>>(p);
+    invl_kernel<F, true, MIRROR><<<grid, kInvlWarps * 32, 0, s>>>(p);
   else
-    invl_kernel<F, false><<<grid, kInvlWarps * 32, 0, s>>>(p);
+    invl_kernel<F, false, MIRROR><<<grid, kInvlWarps * 32, 0, s>>>(p);
   return cudaGetLastError();
 }
 
-cudaError_t launch_invl(int func, const FillParams& p, int grid, cudaStream_t s) {
-  switch (func) {
-    case 4: return launch_il<CellDiagMaxPlus>(p, grid, s);
-    default: return cudaErrorInvalidValue;
-  }
+// func 4 DIAG_MAXPLUS (Inverted-L) and 8 ANTIDIAG_MAXPLUS (its mirror twin, the same cell on the
+// mirrored grid, mirror = true)
+cudaError_t launch_invl(int func, const FillParams& p, int grid, bool mirror, cudaStream_t s) {
+  if (func != 4 && func != 8) return cudaErrorInvalidValue;
+  return mirror ? launch_il<CellDiagMaxPlus, true>(p, grid, s) : launch_il<CellDiagMaxPlus, false>(p, grid, s);
 }
 
 }  // namespace lddp

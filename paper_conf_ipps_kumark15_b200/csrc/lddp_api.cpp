@@ -90,6 +90,8 @@ uint32_t category_allows(int cat) {
     case LDDP_CAT_ANTI_DIAGONAL: return LDDP_NB_L | LDDP_NB_UL | LDDP_NB_U;
     case LDDP_CAT_KNIGHT_MOVE: return LDDP_NB_L | LDDP_NB_UL | LDDP_NB_U | LDDP_NB_UR;
     case LDDP_CAT_INVERTED_L: return LDDP_NB_UL;
+    case LDDP_CAT_VERTICAL: return LDDP_NB_L | LDDP_NB_UL;     // t = j: L (t-1), UL (t-1)
+    case LDDP_CAT_MINVERTED_L: return LDDP_NB_UR;              // t = min(i, W-1-j): UR only
     default: return 0;
   }
 }
@@ -103,6 +105,8 @@ uint32_t func_mask(int f) {
     case LDDP_F_DIAG_MAXPLUS: return LDDP_NB_UL;
     case LDDP_F_MIN2_PLUS: return LDDP_NB_UL | LDDP_NB_U;
     case LDDP_F_LEVENSHTEIN: return LDDP_NB_L | LDDP_NB_UL | LDDP_NB_U;
+    case LDDP_F_MIN2_PLUS_V: return LDDP_NB_L | LDDP_NB_UL;
+    case LDDP_F_ANTIDIAG_MAXPLUS: return LDDP_NB_UR;
     default: return 0;
   }
 }
@@ -213,6 +217,11 @@ struct lddp_plan_s {
   int cb_nblocks;    // column blocks (one warp each)
   // Floyd-Steinberg lane-systolic kernel (fsk.cu): used when the widths / pitches allow
   bool fsk;
+  // symmetric twins: mInverted-L = the inverted-L kernel on the mirrored grid; Vertical = a
+  // transpose + the prev-row plan of the transposed problem (inner), workspace offsets below
+  bool mirror;
+  lddp_plan_s* inner;
+  size_t off_tab, off_inner;
   int fsk_W, fsk_E, fsk_R, fsk_nstrips;
   int64_t fsk_bnd_stride;
   // workspace layout (bytes)
@@ -424,8 +433,36 @@ lddp_status launch(lddp_plan_t pl, const FillParams& p, cudaStream_t s) {
       if (const char* g = getenv("LDDP_PREVROW_CTAS")) grid = std::max(1, atoi(g) / 2);
     }
     e = lddp::launch_prevrow(pl->desc.func, q, grid, s);
+  } else if (pl->kind == 5) {
+    // Vertical: grid (H x W) -> workspace (W x H), the transposed prev-row fill, table back
+    lddp_plan_s* in = pl->inner;
+    char* ws = static_cast<char*>(p.ctl);
+    const int64_t H = pl->desc.rows, W = pl->desc.cols;
+    int32_t* tg = reinterpret_cast<int32_t*>(ws + pl->off_bnd);
+    e = lddp::launch_transpose_i32(static_cast<const int32_t*>(p.grid), p.grid_pitch, tg, H, H, W, s);
+    if (e != cudaSuccess) return cuda_fail(e, "transpose launch");
+    lddp_inputs din{};
+    din.grid = tg;
+    din.grid_pitch = H;
+    lddp_outputs dout{};
+    dout.score = p.score;
+    dout.last_row = p.last_col;
+    int32_t* tt = reinterpret_cast<int32_t*>(ws + pl->off_tab);
+    if (p.table != nullptr) {
+      dout.table = tt;
+      dout.table_pitch = H;
+    }
+    FillParams q;
+    fill_common(in, &din, &dout, ws + pl->off_inner, q);
+    lddp_status st = launch(in, q, s);
+    if (st != LDDP_OK) return st;
+    if (p.table != nullptr) {
+      e = lddp::launch_transpose_i32(tt, H, static_cast<int32_t*>(p.table), p.table_pitch, W, H, s);
+      if (e != cudaSuccess) return cuda_fail(e, "transpose launch");
+    }
+    return LDDP_OK;
   } else {
-    e = lddp::launch_invl(pl->desc.func, p, pl->grid, s);
+    e = lddp::launch_invl(pl->desc.func, p, pl->grid, pl->mirror, s);
   }
   if (e != cudaSuccess) return cuda_fail(e, "kernel launch");
   return LDDP_OK;
@@ -472,7 +509,7 @@ lddp_status lddp_classify(uint32_t mask, int32_t* pattern) {
 
 lddp_status lddp_category_covers(int32_t category, uint32_t mask, int32_t* covers) {
   if (covers == nullptr) return fail(LDDP_ERR_INVALID_ARG, "covers is NULL");
-  if (category < 0 || category > 3) return fail(LDDP_ERR_INVALID_ARG, "unknown category %d", category);
+  if (category < 0 || category > 5) return fail(LDDP_ERR_INVALID_ARG, "unknown category %d", category);
   if (mask == 0 || mask > 15) return fail(LDDP_ERR_INVALID_ARG, "bad mask");
   *covers = (mask & ~category_allows(category)) == 0 ? 1 : 0;
   return LDDP_OK;
@@ -485,7 +522,7 @@ lddp_status lddp_plan(const lddp_desc* desc, lddp_plan_t* out) {
     const lddp_desc& d = *desc;
     const uint32_t fm = func_mask(d.func);
     if (fm == 0) return fail(LDDP_ERR_INVALID_ARG, "unknown func %d", d.func);
-    if (d.category < 0 || d.category > 3) return fail(LDDP_ERR_INVALID_ARG, "unknown category %d", d.category);
+    if (d.category < 0 || d.category > 5) return fail(LDDP_ERR_INVALID_ARG, "unknown category %d", d.category);
     if (d.rows < 0 || d.cols < 0) return fail(LDDP_ERR_SHAPE, "negative shape");
     if (d.cols > (int64_t)0x7fff0000 || d.rows > ((int64_t)1 << 40)) return fail(LDDP_ERR_SHAPE, "shape too large");
     if (d.outputs & ~(LDDP_OUT_SCORE | LDDP_OUT_LAST_ROW | LDDP_OUT_LAST_COL | LDDP_OUT_TABLE))
@@ -500,6 +537,15 @@ lddp_status lddp_plan(const lddp_desc* desc, lddp_plan_t* out) {
       return fail(LDDP_ERR_INVALID_ARG, "f=%d has no score output", d.func);
     if ((d.outputs & LDDP_OUT_LAST_COL) && d.category == LDDP_CAT_PREV_ROW)
       return fail(LDDP_ERR_UNSUPPORTED, "LAST_COL is not produced by the prev-row kernel");
+    // the symmetric twins' f's run only in their own categories (on their twins' kernels)
+    if ((d.func == LDDP_F_MIN2_PLUS_V) != (d.category == LDDP_CAT_VERTICAL) ||
+        (d.func == LDDP_F_ANTIDIAG_MAXPLUS) != (d.category == LDDP_CAT_MINVERTED_L))
+      return fail(LDDP_ERR_UNSUPPORTED, "f=%d in category %d: the twin f's MIN2_PLUS_V / ANTIDIAG_MAXPLUS run in "
+                  "the VERTICAL / MINVERTED_L categories, and only those f's are compiled for them", d.func, d.category);
+    if ((d.outputs & LDDP_OUT_LAST_ROW) && d.category == LDDP_CAT_VERTICAL)
+      return fail(LDDP_ERR_UNSUPPORTED, "LAST_ROW is not produced by the vertical (transposed prev-row) path");
+    if ((d.outputs & LDDP_OUT_SCORE) && d.func == LDDP_F_ANTIDIAG_MAXPLUS)
+      return fail(LDDP_ERR_INVALID_ARG, "f=%d has no score output", d.func);
     if (d.func == LDDP_F_MIN_PATH3 && d.rows == 0 && d.cols > 0)
       return fail(LDDP_ERR_SHAPE, "MIN_PATH3 needs at least one row");
 
@@ -693,8 +739,33 @@ lddp_status lddp_plan(const lddp_desc* desc, lddp_plan_t* out) {
           cudaGetLastError();
         }
       }
+    } else if (d.category == LDDP_CAT_VERTICAL) {
+      // Vertical = transpose of Horizontal [L111]: transpose the grid into the workspace, run the
+      // prev-row plan of the transposed problem (its last row = our last column, its score =
+      // ours), transpose a TABLE output back
+      pl->kind = 5;
+      lddp_desc t = d;
+      t.rows = d.cols;
+      t.cols = d.rows;
+      t.category = LDDP_CAT_PREV_ROW;
+      t.func = LDDP_F_MIN2_PLUS;
+      t.outputs = (d.outputs & LDDP_OUT_SCORE) | ((d.outputs & LDDP_OUT_LAST_COL) ? LDDP_OUT_LAST_ROW : 0u) |
+                  (d.outputs & LDDP_OUT_TABLE);
+      lddp_status st = lddp_plan(&t, &pl->inner);
+      if (st != LDDP_OK) {
+        delete pl;
+        return st;
+      }
+      const size_t cells = (size_t)std::max<int64_t>(d.rows, 0) * (size_t)std::max<int64_t>(d.cols, 0);
+      pl->off_prog = 64;
+      pl->off_bnd = 256;                                             // transposed grid (W x H)
+      pl->off_tab = align_up(pl->off_bnd + cells * 4, 256);          // transposed table (TABLE)
+      pl->off_inner = align_up(pl->off_tab + ((d.outputs & LDDP_OUT_TABLE) ? cells * 4 : 0), 256);
+      pl->ws_bytes = pl->off_inner + std::max<size_t>(pl->inner->ws_bytes, 64);
+      pl->grid = 1;
     } else {
       pl->kind = 2;
+      pl->mirror = d.category == LDDP_CAT_MINVERTED_L;   // mInverted-L = mirror of Inverted-L [L111]
       const int64_t nd = d.rows + d.cols - 1;
       const int64_t warps = (nd + 31) / 32;
       const int64_t blocks = (warps + (kInvlThreads / 32) - 1) / (kInvlThreads / 32);
@@ -712,6 +783,7 @@ lddp_status lddp_plan(const lddp_desc* desc, lddp_plan_t* out) {
 
 lddp_status lddp_plan_destroy(lddp_plan_t pl) {
   if (pl == nullptr) return LDDP_OK;
+  if (pl->inner) lddp_plan_destroy(pl->inner);
   DeviceGuard dg(pl->desc.device);
   if (pl->own_ws) cudaFree(pl->own_ws);
   for (int k = 0; k < 6; ++k)
@@ -728,7 +800,13 @@ lddp_status lddp_plan_workspace_size(lddp_plan_t pl, size_t* bytes) {
 
 lddp_status lddp_plan_describe(lddp_plan_t pl, char* buf, size_t len) {
   if (pl == nullptr || buf == nullptr || len == 0) return fail(LDDP_ERR_INVALID_ARG, "NULL argument");
-  static const char* kinds[] = {"wavefront", "prevrow", "invl", "adiag", "lcs16"};
+  static const char* kinds[] = {"wavefront", "prevrow", "invl", "adiag", "lcs16", "transpose+prevrow"};
+  if (pl->kind == 5) {   // Vertical twin: describe the transposed prev-row plan it runs
+    char inner[768];
+    lddp_plan_describe(pl->inner, inner, sizeof inner);
+    snprintf(buf, len, "{\"kernel\": \"transpose+prevrow\", \"workspace_bytes\": %zu, \"inner\": %s}", pl->ws_bytes, inner);
+    return LDDP_OK;
+  }
   const bool cb = pl->kind == 1 && pl->cb_variant >= 0;
   if (pl->kind == 0 && pl->fsk) {
     snprintf(buf, len,
@@ -744,13 +822,14 @@ lddp_status lddp_plan_describe(lddp_plan_t pl, char* buf, size_t len) {
   snprintf(buf, len,
            "{\"kernel\": \"%s\", \"variant\": %d, \"rows_per_lane\": %d, \"skew\": %d, \"extra_lag\": %d, "
            "\"warps\": %d, \"grid\": %d, \"sms\": %d, \"occupancy\": %d, \"strip_rows\": %lld, "
-           "\"strips\": %d, \"chunks\": %d, \"blocks\": %d, \"bands\": %d, \"workspace_bytes\": %zu}",
+           "\"strips\": %d, \"chunks\": %d, \"blocks\": %d, \"bands\": %d, \"workspace_bytes\": %zu, "
+           "\"mirror\": %d}",
            cb ? "prevrow_cb" : kinds[pl->kind], cb ? pl->cb_variant : pl->variant, pl->R, pl->SIG, pl->E,
            cb ? pl->cb_nw
               : (pl->kind == 0 ? kWfWarps + 2 : (pl->kind == 1 ? kPrevThreads / 32 : (pl->kind >= 3 ? pl->W : kInvlThreads / 32))),
            cb ? (pl->cb_nblocks + pl->cb_nw - 1) / pl->cb_nw : pl->grid,
            pl->sms, cb ? 1 : pl->occupancy, (long long)pl->strip_rows, pl->nstrips, pl->nchunks,
-           cb ? pl->cb_nblocks : pl->nblocks, pl->nbands, pl->ws_bytes);
+           cb ? pl->cb_nblocks : pl->nblocks, pl->nbands, pl->ws_bytes, pl->mirror ? 1 : 0);
   return LDDP_OK;
 }
 

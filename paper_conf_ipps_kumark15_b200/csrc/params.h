@@ -71,7 +71,12 @@ cudaError_t launch_fsk(const FillParams& p, int W, int E, int R, int grid, cudaS
 // Traceback of a LCS / Levenshtein / DTW table (traceback.cu): one thread, O(m + n).
 cudaError_t launch_traceback(int func, const void* a, const void* b, const void* table, int64_t pitch, int64_t m,
                              int64_t n, int32_t* pi, int32_t* pj, int64_t* len, cudaStream_t s);
-cudaError_t launch_invl(int func, const FillParams& p, int grid, cudaStream_t stream);
+// Inverted-L kernel (invl.cu); mirror: read / write the grid with column j <-> W-1-j (the
+// mInverted-L twin [L111]).
+cudaError_t launch_invl(int func, const FillParams& p, int grid, bool mirror, cudaStream_t stream);
+// dst (cols x rows) = transpose of src (rows x cols), 32-bit elements, pitches in elements.
+cudaError_t launch_transpose_i32(const int32_t* src, int64_t spitch, int32_t* dst, int64_t dpitch, int64_t rows,
+                                 int64_t cols, cudaStream_t s);
 // Packed 16x2 LCS kernel (lcs16.cu): P row pairs per lane (strips of 64P rows), lane lag E.
 cudaError_t launch_lcs16(const FillParams& p, int P, int E, int grid, cudaStream_t stream);
 bool lcs16_compiled(int P, int E);

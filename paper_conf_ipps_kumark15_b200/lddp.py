@@ -30,14 +30,17 @@ STATUS_NAMES = {0: "LDDP_OK", 1: "LDDP_ERR_INVALID_ARG", 2: "LDDP_ERR_SHAPE",
 LDDP_ERR_INVALID_ARG, LDDP_ERR_SHAPE, LDDP_ERR_CATEGORY_MISMATCH, LDDP_ERR_UNSUPPORTED = 1, 2, 3, 4
 LDDP_ERR_TIMEOUT = 8
 
-CAT_PREV_ROW, CAT_ANTI_DIAGONAL, CAT_KNIGHT_MOVE, CAT_INVERTED_L = 0, 1, 2, 3
-CATEGORIES = {"prev_row": 0, "anti_diagonal": 1, "knight_move": 2, "inverted_l": 3}
+CAT_PREV_ROW, CAT_ANTI_DIAGONAL, CAT_KNIGHT_MOVE, CAT_INVERTED_L, CAT_VERTICAL, CAT_MINVERTED_L = range(6)
+CATEGORIES = {"prev_row": 0, "anti_diagonal": 1, "knight_move": 2, "inverted_l": 3, "vertical": 4,
+              "minverted_l": 5}
 PAT_HORIZONTAL, PAT_ANTI_DIAGONAL, PAT_KNIGHT_MOVE, PAT_INVERTED_L, PAT_VERTICAL, PAT_MINVERTED_L = range(6)
 PATTERN_NAMES = {0: "Horizontal", 1: "Anti-diagonal", 2: "Knight-Move", 3: "Inverted-L",
                  4: "Vertical", 5: "mInverted-L"}
 NB_L, NB_UL, NB_U, NB_UR = 1, 2, 4, 8
-F_LCS, F_DTW, F_FS_DITHER, F_MIN_PATH3, F_DIAG_MAXPLUS, F_MIN2_PLUS, F_LEVENSHTEIN = range(7)
-FUNCS = {"lcs": 0, "dtw": 1, "fs": 2, "minpath3": 3, "diagmaxplus": 4, "min2plus": 5, "levenshtein": 6}
+(F_LCS, F_DTW, F_FS_DITHER, F_MIN_PATH3, F_DIAG_MAXPLUS, F_MIN2_PLUS, F_LEVENSHTEIN, F_MIN2_PLUS_V,
+ F_ANTIDIAG_MAXPLUS) = range(9)
+FUNCS = {"lcs": 0, "dtw": 1, "fs": 2, "minpath3": 3, "diagmaxplus": 4, "min2plus": 5, "levenshtein": 6,
+         "min2plus_v": 7, "antidiag_maxplus": 8}
 OUT_SCORE, OUT_LAST_ROW, OUT_LAST_COL, OUT_TABLE = 1, 2, 4, 8
 COMM_HANDLE_BYTES = 64
 

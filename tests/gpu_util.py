@@ -8,7 +8,7 @@ OUT_DTYPE = {"lcs": np.int32, "levenshtein": np.int32, "dtw": np.float32, "fs": 
 
 
 def run_gpu(func, category, *, a=None, b=None, grid=None, outputs=("score", "last_row"),
-            param_c=1, tile_rows=0, grid_ctas=0, table_pad=0, reps=1):
+            param_c=1, tile_rows=0, grid_ctas=0, table_pad=0, reps=1, grid_pad=0):
     import torch
 
     from paper_conf_ipps_kumark15_b200 import lddp
@@ -33,8 +33,8 @@ def run_gpu(func, category, *, a=None, b=None, grid=None, outputs=("score", "las
         t["b"] = torch.from_numpy(np.ascontiguousarray(b)).to(dev)
     else:
         g = np.ascontiguousarray(grid)
-        if func == "fs" and cols % 4:
-            pad = np.zeros((rows, cols + (-cols) % 4), g.dtype)
+        if (func == "fs" and cols % 4) or grid_pad:
+            pad = np.zeros((rows, cols + (-cols) % 4 + grid_pad), g.dtype)   # row pitch > cols
             pad[:, :cols] = g
             t["grid"] = torch.from_numpy(pad).to(dev)[:, :cols]
         else:

@@ -52,7 +52,8 @@ def test_classify_matches_table1(lddp):
         assert lddp.lddp_classify(mask) == names[row["pattern"]], row
 
 
-CAT_PATTERN = {0: "Horizontal", 1: "Anti-diagonal", 2: "Knight-Move", 3: "Inverted-L"}
+CAT_PATTERN = {0: "Horizontal", 1: "Anti-diagonal", 2: "Knight-Move", 3: "Inverted-L", 4: "Vertical",
+               5: "mInverted-L"}
 
 
 def test_category_covers_matches_schedules(lddp):
@@ -71,6 +72,11 @@ def test_func_masks(lddp):
     assert lddp.lddp_func_mask(lddp.F_MIN_PATH3) == 2 | 4 | 8    # [L365]
     assert lddp.lddp_func_mask(lddp.F_DIAG_MAXPLUS) == 2         # [L298]
     assert lddp.lddp_func_mask(lddp.F_MIN2_PLUS) == 2 | 4        # [L298]
+    assert lddp.lddp_func_mask(lddp.F_MIN2_PLUS_V) == 1 | 2      # Vertical twin [L111], R15
+    assert lddp.lddp_func_mask(lddp.F_ANTIDIAG_MAXPLUS) == 8     # mInverted-L twin [L111], R15
+    # Table I classifies each compiled f into the pattern of the category it runs in
+    assert lddp.lddp_classify(lddp.lddp_func_mask(lddp.F_MIN2_PLUS_V)) == lddp.PAT_VERTICAL
+    assert lddp.lddp_classify(lddp.lddp_func_mask(lddp.F_ANTIDIAG_MAXPLUS)) == lddp.PAT_MINVERTED_L
     with pytest.raises(lddp.LddpError):
         lddp.lddp_func_mask(99)
 
@@ -87,6 +93,16 @@ def test_plan_rejects_category_mismatch_without_gpu(lddp):
     with pytest.raises(lddp.LddpError) as e:
         lddp.lddp_plan(d)
     assert e.value.status == lddp.LDDP_ERR_CATEGORY_MISMATCH
+    for cat, func in ((lddp.CAT_INVERTED_L, lddp.F_ANTIDIAG_MAXPLUS), (lddp.CAT_PREV_ROW, lddp.F_MIN2_PLUS_V)):
+        d = lddp.lddp_desc(rows=10, cols=10, category=cat, func=func, outputs=lddp.OUT_LAST_ROW)
+        with pytest.raises(lddp.LddpError) as e:   # {UR} / {L,UL} not ordered by these schedules
+            lddp.lddp_plan(d)
+        assert e.value.status == lddp.LDDP_ERR_CATEGORY_MISMATCH
+    d = lddp.lddp_desc(rows=10, cols=10, category=lddp.CAT_ANTI_DIAGONAL, func=lddp.F_MIN2_PLUS_V,
+                       outputs=lddp.OUT_SCORE)
+    with pytest.raises(lddp.LddpError) as e:       # ordered, but the twin f runs on its twin's kernel
+        lddp.lddp_plan(d)
+    assert e.value.status == lddp.LDDP_ERR_UNSUPPORTED
     d = lddp.lddp_desc(rows=-1, cols=10, category=lddp.CAT_ANTI_DIAGONAL, func=lddp.F_LCS,
                        outputs=lddp.OUT_SCORE)
     with pytest.raises(lddp.LddpError) as e:
