@@ -267,6 +267,7 @@ struct CellMin2Plus {
 // [L298] §V.B Inverted-L synthetic f = max(cell_{i,j}, f(i-1,j-1)) + c, cell = init (reading
 // R9); row 0 and column 0 are init.
 struct CellDiagMaxPlus {
+  static constexpr bool kDirectGrid = true;   // invl.cuh streams the grid with a running pointer
   using T = int32_t;
   using RowCtx = int32_t;
   using ColCtx = int32_t;
