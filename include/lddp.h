@@ -140,7 +140,9 @@ typedef struct {
     int32_t device;          /* CUDA device ordinal the plan is bound to                        */
     int32_t tile_rows;       /* tuning: rows per lane (anti-diagonal / knight), 0 = auto        */
     int32_t tile_warps;      /* tuning: compute warps per CTA, 0 = auto                         */
-    int32_t band_rows;       /* tuning: rows per band (prev-row category), 0 = auto             */
+    int32_t band_rows;       /* tuning, prev-row category: trapezoid band height HB (rows between
+                                two halo exchanges of the column-block kernel): 16, 32, 48 or
+                                64 (else LDDP_ERR_UNSUPPORTED); 0 = auto (32)                    */
     int32_t grid_ctas;       /* tuning: persistent grid size, 0 = auto (SMs x occupancy)        */
     int32_t reserved[3];     /* must be 0                                                       */
 } lddp_desc;

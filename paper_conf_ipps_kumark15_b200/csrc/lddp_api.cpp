@@ -717,7 +717,21 @@ lddp_status lddp_plan(const lddp_desc* desc, lddp_plan_t* out) {
       // Column-block persistent kernel: every block co-resident (cooperative launch), W % 4 == 0
       // (16-byte cost segments; the row pitch / base alignment is checked per fill).
       pl->cb_variant = -1;
-      const int cbv = env_int("LDDP_CB_VARIANT", 5);
+      // desc.band_rows = the trapezoid band height HB (rows between two halo exchanges): each
+      // value maps to the compiled column-block geometry with that HB
+      int cbv_def = 5;
+      if (d.band_rows > 0) {
+        const int hb[][2] = {{16, 13}, {32, 5}, {48, 17}, {64, 0}};
+        cbv_def = -2;
+        for (const auto& x : hb)
+          if (x[0] == d.band_rows) cbv_def = x[1];
+        if (cbv_def == -2) {
+          delete pl;
+          return fail(LDDP_ERR_UNSUPPORTED, "band_rows=%d: compiled prev-row band heights are 16, 32, 48, 64",
+                      d.band_rows);
+        }
+      }
+      const int cbv = env_int("LDDP_CB_VARIANT", cbv_def);
       const int cbnw = std::max(1, std::min(8, env_int("LDDP_CB_WARPS", 4)));
       if (cbv >= 0 && d.cols > 0 && d.rows > 0 && d.cols % 4 == 0) {
         int q[2] = {0, 0};

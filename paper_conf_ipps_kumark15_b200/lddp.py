@@ -226,7 +226,7 @@ class Plan:
     """A plan plus its workspace (torch uint8 tensor on the plan's device)."""
 
     def __init__(self, func, category, rows, cols, outputs, param_c=1, device=0, tile_rows=0,
-                 grid_ctas=0):
+                 grid_ctas=0, band_rows=0):
         import torch
         self.func = FUNCS[func] if isinstance(func, str) else int(func)
         self.category = CATEGORIES[category] if isinstance(category, str) else int(category)
@@ -234,7 +234,7 @@ class Plan:
         self.device = int(device)
         self.desc = lddp_desc(rows=self.rows, cols=self.cols, category=self.category, func=self.func,
                               outputs=self.outputs, param_c=int(param_c), device=self.device,
-                              tile_rows=int(tile_rows), tile_warps=0, band_rows=0,
+                              tile_rows=int(tile_rows), tile_warps=0, band_rows=int(band_rows),
                               grid_ctas=int(grid_ctas))
         self.handle = lddp_plan(self.desc)
         self.ws_bytes = lddp_plan_workspace_size(self.handle)

@@ -8,7 +8,7 @@ OUT_DTYPE = {"lcs": np.int32, "levenshtein": np.int32, "dtw": np.float32, "fs": 
 
 
 def run_gpu(func, category, *, a=None, b=None, grid=None, outputs=("score", "last_row"),
-            param_c=1, tile_rows=0, grid_ctas=0, table_pad=0, reps=1, grid_pad=0):
+            param_c=1, tile_rows=0, grid_ctas=0, table_pad=0, reps=1, grid_pad=0, band_rows=0):
     import torch
 
     from paper_conf_ipps_kumark15_b200 import lddp
@@ -24,7 +24,7 @@ def run_gpu(func, category, *, a=None, b=None, grid=None, outputs=("score", "las
     for o in outputs:
         bits |= names[o]
     plan = lddp.Plan(func, category, rows, cols, bits, param_c=param_c, tile_rows=tile_rows,
-                     grid_ctas=grid_ctas)
+                     grid_ctas=grid_ctas, band_rows=band_rows)
     vdt = {np.int32: torch.int32, np.float32: torch.float32}
     cell_dt = torch.float32 if func == "dtw" else torch.int32
     t = {}

@@ -80,3 +80,23 @@ def test_cb_disabled_falls_back(cb_env):
     assert json.loads(got["plan"])["kernel"] == "prevrow"
     assert got["score"] == ref.score
     np.testing.assert_array_equal(got["last_row"], ref.last_row)
+
+
+@pytest.mark.parametrize("band_rows,variant", [(16, 13), (32, 5), (48, 17), (64, 0)])
+@pytest.mark.parametrize("func", ["minpath3", "min2plus"])
+def test_band_rows_selects_band_height(band_rows, variant, func):
+    """lddp_desc.band_rows = the trapezoid band height HB of the column-block kernel."""
+    H, W = 1000, 1536
+    g = inputs.gen_costs(band_rows + H, H, W) if func == "minpath3" else inputs.gen_init(band_rows, H, W)
+    ref = oracle.minpath3(g) if func == "minpath3" else oracle.min2plus(g, 1)
+    got = run_gpu(func, "prev_row", grid=g, outputs=("score", "last_row"), band_rows=band_rows)
+    assert f'"kernel": "prevrow_cb", "variant": {variant},' in got["plan"], got["plan"]
+    assert got["score"] == ref.score
+    np.testing.assert_array_equal(got["last_row"], ref.last_row)
+
+
+def test_band_rows_unsupported_height():
+    from paper_conf_ipps_kumark15_b200 import lddp
+    with pytest.raises(lddp.LddpError) as e:
+        lddp.Plan("minpath3", "prev_row", 100, 128, lddp.OUT_SCORE, band_rows=40)
+    assert e.value.status == lddp.LDDP_ERR_UNSUPPORTED
