@@ -41,16 +41,18 @@ __global__ void __launch_bounds__(kInvlWarps * 32) invl_kernel(const FillParams 
   const int lane = threadIdx.x & 31;
   const int64_t H = p.rows;
   const int W = p.cols;
-  const int64_t nd = H + W - 1;                      // diagonals d = j - i in [-(H-1), W-1]
-  const int64_t nwarps_total = (nd + 31) / 32;
+  // this launch's diagonals d = j - i in [diag_lo, diag_hi) (all of [-(H-1), W-1] on one GPU;
+  // a contiguous share per rank for lddp_fill_multi: the chains are independent, no exchange)
+  const int64_t dlo0 = p.diag_lo, dhi0 = p.diag_hi;
+  const int64_t nwarps_total = (dhi0 - dlo0 + 31) / 32;
   const int64_t gw0 = (int64_t)blockIdx.x * kInvlWarps + (threadIdx.x >> 5);
   const int64_t gstride = (int64_t)gridDim.x * kInvlWarps;
   for (int64_t gw = gw0; gw < nwarps_total; gw += gstride) {
-    const int64_t d = -(H - 1) + gw * 32 + lane;     // this lane's diagonal
-    const bool live = d <= (int64_t)W - 1;
+    const int64_t d = dlo0 + gw * 32 + lane;         // this lane's diagonal
+    const bool live = d < dhi0;
     // rows this warp visits: union of its lanes' chains
-    const int64_t dlo = -(H - 1) + gw * 32;
-    const int64_t dhi = min((int64_t)W - 1, dlo + 31);
+    const int64_t dlo = dlo0 + gw * 32;
+    const int64_t dhi = min(dhi0 - 1, dlo + 31);
     const int64_t ibeg = max((int64_t)0, -dhi);
     const int64_t iend = min(H, (int64_t)W - dlo);   // exclusive
     // this lane's chain: rows [ia, ib)

@@ -370,6 +370,8 @@ void fill_common(lddp_plan_t pl, const lddp_inputs* in, const lddp_outputs* out,
   p.debug = env_int("LDDP_DEBUG", 0);
   p.spin_polls = env_int("LDDP_SPIN", 256);
   p.one = 1;
+  p.diag_lo = -(d.rows - 1);
+  p.diag_hi = d.cols;
   // debug trace buffer: LDDP_TRACE=<device pointer as decimal>:<chunks per row>
   if (const char* tr = getenv("LDDP_TRACE")) {
     unsigned long long ptr = 0;
@@ -983,9 +985,11 @@ lddp_status lddp_multi_partition(int64_t cols, int32_t nranks, int32_t rank, int
 lddp_status lddp_comm_create(lddp_plan_t pl, int32_t nranks, int32_t rank, lddp_comm_t* out) {
   if (pl == nullptr || out == nullptr) return fail(LDDP_ERR_INVALID_ARG, "NULL argument");
   if (nranks < 1 || rank < 0 || rank >= nranks) return fail(LDDP_ERR_INVALID_ARG, "bad rank %d / %d", rank, nranks);
-  if ((pl->kind != 3 && pl->kind != 4) || pl->desc.category != LDDP_CAT_ANTI_DIAGONAL)
-    return fail(LDDP_ERR_UNSUPPORTED, "multi-GPU column strips: anti-diagonal LCS / Levenshtein / DTW (no TABLE)");
-  if (pl->desc.cols < nranks) return fail(LDDP_ERR_SHAPE, "cols < nranks");
+  const bool chains = pl->kind == 2;   // inverted-L / mInverted-L: diagonal shares, no exchange
+  if (!chains && ((pl->kind != 3 && pl->kind != 4) || pl->desc.category != LDDP_CAT_ANTI_DIAGONAL))
+    return fail(LDDP_ERR_UNSUPPORTED, "multi-GPU: anti-diagonal LCS / Levenshtein / DTW (column strips) or "
+                "inverted-L / mInverted-L (diagonal shares)");
+  if (!chains && pl->desc.cols < nranks) return fail(LDDP_ERR_SHAPE, "cols < nranks");
   DeviceGuard dg(pl->desc.device);
   lddp_comm_s* c = new (std::nothrow) lddp_comm_s();
   if (c == nullptr) return fail(LDDP_ERR_OUT_OF_MEMORY, "comm allocation");
@@ -1124,14 +1128,47 @@ lddp_status lddp_fill_multi(lddp_plan_t pl, const lddp_inputs* in, const lddp_ou
     if (c->plan != pl) return fail(LDDP_ERR_INVALID_ARG, "comm was created for another plan");
     lddp_status st = check_inputs(pl, in, out);
     if (st != LDDP_OK) return st;
-    if (c->rank < c->nranks - 1 && c->next == nullptr)
+    if (pl->kind != 2 && c->rank < c->nranks - 1 && c->next == nullptr)
       return fail(LDDP_ERR_COMM, "rank %d is not connected to rank %d", c->rank, c->rank + 1);
-    if (c->rank > 0 && c->prev == nullptr)
+    if (pl->kind != 2 && c->rank > 0 && c->prev == nullptr)
       return fail(LDDP_ERR_COMM, "rank %d is not connected to rank %d", c->rank, c->rank - 1);
-    if (pl->desc.outputs & LDDP_OUT_TABLE) return fail(LDDP_ERR_UNSUPPORTED, "TABLE output is not supported by lddp_fill_multi");
     DeviceGuard dg(pl->desc.device);
     cudaStream_t s = (cudaStream_t)stream;
     const lddp_desc& d = pl->desc;
+    if (pl->kind == 2) {
+      // Inverted-L (and its mirror twin): every diagonal chain is independent ([L203]); rank g
+      // fills a contiguous share of the diagonals holding ~1/P of the cells, writing its chains'
+      // ends into last_row / last_col and its cells into a TABLE output.  No communication.
+      if (d.rows == 0 || d.cols == 0) return LDDP_OK;
+      st = ensure_own_ws(pl, &ws, s);
+      if (st != LDDP_OK) return st;
+      FillParams p;
+      fill_common(pl, in, out, ws, p);
+      const int64_t H = d.rows, W = d.cols;
+      auto len = [&](int64_t dd) { return std::min(H, W - dd) - std::max<int64_t>(0, -dd); };
+      const double total = (double)H * (double)W;
+      const double lo_target = total * c->rank / c->nranks, hi_target = total * (c->rank + 1) / c->nranks;
+      double acc = 0.0;
+      int64_t dlo = -(H - 1), dhi = W;
+      bool have_lo = c->rank == 0;
+      for (int64_t dd = -(H - 1); dd < W; ++dd) {
+        if (!have_lo && acc >= lo_target) { dlo = dd; have_lo = true; }
+        acc += (double)len(dd);
+        if (c->rank < c->nranks - 1 && acc >= hi_target) { dhi = dd + 1; break; }
+      }
+      if (!have_lo) dlo = W;
+      p.diag_lo = dlo;
+      p.diag_hi = std::max(dlo, dhi);
+      c->fills += 1;
+      if (p.diag_hi == p.diag_lo) return LDDP_OK;
+      const int64_t warps = (p.diag_hi - p.diag_lo + 31) / 32;
+      const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((warps + kInvlThreads / 32 - 1) / (kInvlThreads / 32),
+                                                                   (int64_t)pl->sms * 16));
+      cudaError_t e = lddp::launch_invl(d.func, p, grid, pl->mirror, s);
+      if (e != cudaSuccess) return cuda_fail(e, "kernel launch");
+      return LDDP_OK;
+    }
+    if (pl->desc.outputs & LDDP_OUT_TABLE) return fail(LDDP_ERR_UNSUPPORTED, "TABLE output is not supported by lddp_fill_multi");
     if (d.rows == 0) return LDDP_OK;
     st = ensure_own_ws(pl, &ws, s);
     if (st != LDDP_OK) return st;

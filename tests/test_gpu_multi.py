@@ -192,3 +192,37 @@ def test_cross_process_ipc(func, world):
         score = parts[-1][3][k][0]
         lcol = np.asarray(parts[-1][3][k][2], ref.last_col.dtype)
         _check(func, (np.asarray(score, ref.last_row.dtype), last, lcol), ref)
+
+
+# ------------------------------------------------------------------ inverted-L diagonal shares
+@pytest.mark.parametrize("func,cat", [("diagmaxplus", "inverted_l"), ("antidiag_maxplus", "minverted_l")])
+@pytest.mark.parametrize("P", [1, 2, 3, 8])
+@pytest.mark.parametrize("shape", [(1, 1), (700, 900), (1537, 100), (64, 3000)])
+def test_inverted_l_diagonal_shares(func, cat, P, shape):
+    """Inverted-L chains are independent ([L203]): each rank fills a contiguous share of the
+    diagonals (equal cells), no window traffic; the union of the ranks' outputs equals the oracle."""
+    import torch
+
+    from paper_conf_ipps_kumark15_b200 import lddp
+    H, W = shape
+    g = inputs.gen_init(H + 3 * W + P, H, W)
+    ref = (oracle.diagmaxplus if func == "diagmaxplus" else oracle.antidiag_maxplus)(g, 1, table=True)
+    dev = torch.device("cuda:0")
+    plan = lddp.Plan(func, cat, H, W, lddp.OUT_LAST_ROW | lddp.OUT_LAST_COL | lddp.OUT_TABLE)
+    comms = [lddp.lddp_comm_create(plan.handle, P, r) for r in range(P)]
+    tg = torch.from_numpy(g).to(dev)
+    lr = torch.full((W,), -7, dtype=torch.int32, device=dev)
+    lc = torch.full((H,), -7, dtype=torch.int32, device=dev)
+    tab = torch.full((H, W), -7, dtype=torch.int32, device=dev)
+    wss = [torch.zeros(max(plan.ws_bytes, 64), dtype=torch.uint8, device=dev) for _ in range(P)]
+    try:
+        for r in range(P):   # no connect needed: no exchange
+            inp, out = plan.io(grid=tg, last_row=lr, last_col=lc, table=tab)
+            lddp.lddp_fill_multi(plan.handle, inp, out, wss[r].data_ptr(), comms[r], 0)
+        torch.cuda.synchronize()
+        np.testing.assert_array_equal(tab.cpu().numpy(), ref.table)
+        np.testing.assert_array_equal(lr.cpu().numpy(), ref.last_row)
+        np.testing.assert_array_equal(lc.cpu().numpy(), ref.last_col)
+    finally:
+        for c in comms:
+            lddp.lddp_comm_destroy(c)
