@@ -231,7 +231,19 @@ lddp_status lddp_status_check(lddp_plan_t plan, void* workspace, void* stream);
  * finished row strip straight into rank g+1's receive window over NVLink (peer stores + a
  * system-scope release flag per strip: the one-way boundary transfer of Table II's
  * anti-diagonal row [L265-L274], [L164]) and reads rank g-1's column from its own window.
- * Supported for the anti-diagonal category (LCS, Levenshtein, DTW) in this build.
+ * Supported categories:
+ *   anti-diagonal (LCS, Levenshtein, DTW): column strips, one-way boundary transfer (above);
+ *   previous-row (min-path, min2plus; cols % 4 == 0): column strips made of whole column blocks
+ *     of the column-block kernel (lddp_plan_partition); every HB-row band the strip's outer
+ *     blocks store their HB edge columns into the neighbour ranks' windows as tagged (value,
+ *     fill epoch | band) pairs and read the neighbours' edges from their own window -- the
+ *     two-way trapezoid halo of Table II case 2 [L265-L274], [L193-L195].  Window halo region:
+ *     [from g-1: 8 slots][from g+1: 8 slots] x 64 pairs, slot = (fill parity, band mod 4).
+ *     Every rank's kernel must be resident at once (they exchange every band).  Rank g writes
+ *     last_row / table columns [c0, c1) and score = the minimum of ITS last-row columns (the
+ *     global score is the minimum over ranks);
+ *   inverted-L / mInverted-L: diagonal shares d = j - i in [lo, hi) holding ~1/P of the cells
+ *     (every chain independent [L203]): no exchange; rank g writes its chains' cells and ends.
  *
  * Window of rank g (device memory of rank g), two slots selected by fill parity so that fill
  * k+1 can start on rank g-1 while rank g is still reading fill k:
@@ -254,6 +266,10 @@ lddp_status lddp_status_check(lddp_plan_t plan, void* workspace, void* stream);
 #define LDDP_COMM_HANDLE_BYTES 64
 /* Columns [c0, c1) of rank `rank` of `nranks` for a problem with `cols` columns (host only). */
 lddp_status lddp_multi_partition(int64_t cols, int32_t nranks, int32_t rank, int64_t* c0, int64_t* c1);
+/* The share of rank `rank` of `nranks` in lddp_fill_multi for this plan: columns [lo, hi) for
+ * column strips (anti-diagonal: lddp_multi_partition; prev-row: whole column blocks), diagonals
+ * d = j - i in [lo, hi) for inverted-L shares.  Host only; errors: INVALID_ARG. */
+lddp_status lddp_plan_partition(lddp_plan_t plan, int32_t nranks, int32_t rank, int64_t* lo, int64_t* hi);
 lddp_status lddp_comm_create(lddp_plan_t plan, int32_t nranks, int32_t rank, lddp_comm_t* comm);
 lddp_status lddp_comm_handle(lddp_comm_t comm, uint8_t handle[LDDP_COMM_HANDLE_BYTES]);
 lddp_status lddp_comm_connect(lddp_comm_t comm, const uint8_t* next_handle, const uint8_t* prev_handle);

@@ -213,6 +213,7 @@ struct lddp_plan_s {
   int nblocks;
   int nbands;
   int cb_variant;    // column-block persistent kernel (prevrow_cb.cu): -1 = not usable
+  int cb_bw;         // its own columns per warp (block width)
   int cb_nw;         // warps per CTA
   int cb_nblocks;    // column blocks (one warp each)
   // Floyd-Steinberg lane-systolic kernel (fsk.cu): used when the widths / pitches allow
@@ -239,7 +240,7 @@ struct lddp_comm_s {
   int nranks, rank, device;
   void* window;          // this rank's window (device memory of this rank)
   size_t win_bytes;
-  size_t off_flag, off_val;
+  size_t off_flag, off_val, off_halo;   // off_halo: prev-row edges [from left 8 x 64][from right 8 x 64]
   int64_t nstrips, rows;
   void* next;            // rank+1's window (IPC-opened or in-process), NULL on the last rank
   void* prev;            // rank-1's window, NULL on rank 0
@@ -745,6 +746,7 @@ lddp_status lddp_plan(const lddp_desc* desc, lddp_plan_t* out) {
             pl->cb_variant = cbv;
             pl->cb_nw = cbnw;
             pl->cb_nblocks = (int)nbq;
+            pl->cb_bw = q[0];
             // workspace: row minima (4 B per block) + edge pairs [nb][4][2][HB <= 64] x 8 B
             const size_t prog = align_up(64 + (size_t)nbq * 4, 256);
             pl->off_prog = 64;
@@ -982,13 +984,57 @@ lddp_status lddp_multi_partition(int64_t cols, int32_t nranks, int32_t rank, int
   return LDDP_OK;
 }
 
+// The share of rank `rank` of `nranks` in a multi-GPU fill of this plan: columns [lo, hi) for
+// column strips (anti-diagonal: near-equal; prev-row: whole column blocks of the column-block
+// kernel), diagonals d = j - i in [lo, hi) for inverted-L diagonal shares (~1/P of the cells).
+static void plan_share(lddp_plan_t pl, int32_t nranks, int32_t rank, int64_t* lo, int64_t* hi) {
+  const lddp_desc& d = pl->desc;
+  const int64_t H = d.rows, W = d.cols;
+  if (pl->kind == 2) {
+    auto len = [&](int64_t dd) { return std::min(H, W - dd) - std::max<int64_t>(0, -dd); };
+    const double total = (double)H * (double)W;
+    const double lo_target = total * rank / nranks, hi_target = total * (rank + 1) / nranks;
+    double acc = 0.0;
+    int64_t dlo = -(H - 1), dhi = W;
+    bool have_lo = rank == 0;
+    for (int64_t dd = -(H - 1); dd < W; ++dd) {
+      if (!have_lo && acc >= lo_target) { dlo = dd; have_lo = true; }
+      acc += (double)len(dd);
+      if (rank < nranks - 1 && acc >= hi_target) { dhi = dd + 1; break; }
+    }
+    if (!have_lo) dlo = W;
+    if (H == 0 || W == 0) dlo = dhi = 0;
+    *lo = dlo;
+    *hi = std::max(dlo, dhi);
+  } else if (pl->kind == 1 && pl->cb_variant >= 0) {
+    const int64_t BW = pl->cb_bw;
+    const int64_t NB = (W + BW - 1) / BW;
+    const int64_t b0 = (int64_t)rank * NB / nranks, b1 = (int64_t)(rank + 1) * NB / nranks;
+    *lo = std::min<int64_t>(b0 * BW, W);
+    *hi = std::min<int64_t>(b1 * BW, W);
+  } else {
+    *lo = (int64_t)rank * W / nranks;
+    *hi = (int64_t)(rank + 1) * W / nranks;
+  }
+}
+
+lddp_status lddp_plan_partition(lddp_plan_t pl, int32_t nranks, int32_t rank, int64_t* lo, int64_t* hi) {
+  if (pl == nullptr || lo == nullptr || hi == nullptr) return fail(LDDP_ERR_INVALID_ARG, "NULL argument");
+  if (nranks < 1 || rank < 0 || rank >= nranks) return fail(LDDP_ERR_INVALID_ARG, "bad rank %d / %d", rank, nranks);
+  plan_share(pl, nranks, rank, lo, hi);
+  return LDDP_OK;
+}
+
 lddp_status lddp_comm_create(lddp_plan_t pl, int32_t nranks, int32_t rank, lddp_comm_t* out) {
   if (pl == nullptr || out == nullptr) return fail(LDDP_ERR_INVALID_ARG, "NULL argument");
   if (nranks < 1 || rank < 0 || rank >= nranks) return fail(LDDP_ERR_INVALID_ARG, "bad rank %d / %d", rank, nranks);
   const bool chains = pl->kind == 2;   // inverted-L / mInverted-L: diagonal shares, no exchange
-  if (!chains && ((pl->kind != 3 && pl->kind != 4) || pl->desc.category != LDDP_CAT_ANTI_DIAGONAL))
-    return fail(LDDP_ERR_UNSUPPORTED, "multi-GPU: anti-diagonal LCS / Levenshtein / DTW (column strips) or "
-                "inverted-L / mInverted-L (diagonal shares)");
+  const bool rows = pl->kind == 1;     // prev-row: column strips, two-way trapezoid halos
+  if (rows && pl->cb_variant < 0)
+    return fail(LDDP_ERR_UNSUPPORTED, "multi-GPU prev-row needs the column-block kernel (cols %% 4 == 0)");
+  if (!chains && !rows && ((pl->kind != 3 && pl->kind != 4) || pl->desc.category != LDDP_CAT_ANTI_DIAGONAL))
+    return fail(LDDP_ERR_UNSUPPORTED, "multi-GPU: anti-diagonal LCS / Levenshtein / DTW (column strips), prev-row "
+                "(column strips, two-way halos) or inverted-L / mInverted-L (diagonal shares)");
   if (!chains && pl->desc.cols < nranks) return fail(LDDP_ERR_SHAPE, "cols < nranks");
   DeviceGuard dg(pl->desc.device);
   lddp_comm_s* c = new (std::nothrow) lddp_comm_s();
@@ -1002,7 +1048,8 @@ lddp_status lddp_comm_create(lddp_plan_t pl, int32_t nranks, int32_t rank, lddp_
   c->rows = pl->desc.rows;
   c->off_flag = align_up((size_t)2 * c->nstrips * 8, 256);
   c->off_val = c->off_flag + align_up((size_t)2 * c->nstrips * 8, 256);
-  c->win_bytes = c->off_val + (size_t)2 * (c->rows + 1) * 4;
+  c->off_halo = align_up(c->off_val + (size_t)2 * (c->rows + 1) * 4, 256);
+  c->win_bytes = c->off_halo + (size_t)2 * 8 * 64 * 8;
   cudaError_t e = cudaMalloc(&c->window, c->win_bytes);
   if (e == cudaSuccess) e = cudaMemset(c->window, 0, c->win_bytes);
   if (e != cudaSuccess) {
@@ -1144,27 +1191,55 @@ lddp_status lddp_fill_multi(lddp_plan_t pl, const lddp_inputs* in, const lddp_ou
       if (st != LDDP_OK) return st;
       FillParams p;
       fill_common(pl, in, out, ws, p);
-      const int64_t H = d.rows, W = d.cols;
-      auto len = [&](int64_t dd) { return std::min(H, W - dd) - std::max<int64_t>(0, -dd); };
-      const double total = (double)H * (double)W;
-      const double lo_target = total * c->rank / c->nranks, hi_target = total * (c->rank + 1) / c->nranks;
-      double acc = 0.0;
-      int64_t dlo = -(H - 1), dhi = W;
-      bool have_lo = c->rank == 0;
-      for (int64_t dd = -(H - 1); dd < W; ++dd) {
-        if (!have_lo && acc >= lo_target) { dlo = dd; have_lo = true; }
-        acc += (double)len(dd);
-        if (c->rank < c->nranks - 1 && acc >= hi_target) { dhi = dd + 1; break; }
-      }
-      if (!have_lo) dlo = W;
+      int64_t dlo = 0, dhi = 0;
+      plan_share(pl, c->nranks, c->rank, &dlo, &dhi);
       p.diag_lo = dlo;
-      p.diag_hi = std::max(dlo, dhi);
+      p.diag_hi = dhi;
       c->fills += 1;
       if (p.diag_hi == p.diag_lo) return LDDP_OK;
       const int64_t warps = (p.diag_hi - p.diag_lo + 31) / 32;
       const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((warps + kInvlThreads / 32 - 1) / (kInvlThreads / 32),
                                                                    (int64_t)pl->sms * 16));
       cudaError_t e = lddp::launch_invl(d.func, p, grid, pl->mirror, s);
+      if (e != cudaSuccess) return cuda_fail(e, "kernel launch");
+      return LDDP_OK;
+    }
+    if (pl->kind == 1) {
+      // Previous-row category: rank g owns a block-aligned column strip; the column-block kernel
+      // exchanges its outer edges with the neighbour ranks every band (two-way trapezoid halos,
+      // Table II case 2 [L265-L274]).  The grid is passed whole (the halos read HB columns of
+      // the neighbours' costs); score = the minimum of this rank's last-row columns.
+      if (d.rows == 0 || d.cols == 0) return LDDP_OK;
+      if ((reinterpret_cast<uintptr_t>(in->grid) & 15) || (in->grid_pitch % 4))
+        return fail(LDDP_ERR_UNSUPPORTED, "multi-GPU prev-row: 16-byte aligned grid, pitch %% 4 == 0");
+      st = ensure_own_ws(pl, &ws, s);
+      if (st != LDDP_OK) return st;
+      int64_t c0 = 0, c1 = 0;
+      plan_share(pl, c->nranks, c->rank, &c0, &c1);
+      c->fills += 1;
+      if (c1 <= c0) return LDDP_OK;
+      FillParams p;
+      fill_common(pl, in, out, ws, p);
+      const size_t gel = grid_elt_bytes(d.func), tel = table_elt_bytes(d.func);
+      p.grid = static_cast<const char*>(in->grid) + c0 * gel;
+      p.cols = (int32_t)(c1 - c0);
+      p.col0 = (int32_t)c0;
+      p.cols_total = (int32_t)d.cols;
+      if (p.last_row) p.last_row = static_cast<char*>(p.last_row) + c0 * cell_bytes(d.func);
+      if (p.table) p.table = static_cast<char*>(p.table) + c0 * tel;
+      p.nblocks = (int)((c1 - c0 + pl->cb_bw - 1) / pl->cb_bw);
+      p.wepoch = c->fills;
+      uint64_t* own = reinterpret_cast<uint64_t*>(static_cast<char*>(c->window) + c->off_halo);
+      if (c->rank > 0) {
+        p.halo_in_l = own;                                                                   // from left
+        p.halo_out_l = reinterpret_cast<uint64_t*>(static_cast<char*>(c->prev) + c->off_halo) + 8 * 64;   // its "from right"
+      }
+      if (c->rank < c->nranks - 1) {
+        p.halo_in_r = own + 8 * 64;                                                          // from right
+        p.halo_out_r = reinterpret_cast<uint64_t*>(static_cast<char*>(c->next) + c->off_halo);            // its "from left"
+      }
+      int dummy2[2];
+      cudaError_t e = lddp::launch_prevrow_cb(d.func, pl->cb_variant, p, pl->cb_nw, false, dummy2, s);
       if (e != cudaSuccess) return cuda_fail(e, "kernel launch");
       return LDDP_OK;
     }

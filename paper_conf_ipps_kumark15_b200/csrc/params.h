@@ -57,6 +57,12 @@ struct FillParams {
   int32_t debug;            // env LDDP_DEBUG bits (development): 1 = adiag warps without handoffs
   int32_t workers;          // lcs16: persistent strip workers (warps); extra warps of the last CTA idle
   int64_t diag_lo, diag_hi; // inverted-L: this rank's diagonals d = j - i in [diag_lo, diag_hi)
+  // prev-row multi-GPU (column strips with two-way trapezoid halos, Table II case 2): edge pairs
+  // [8 slots: fill parity x band mod 4][HB] exchanged with the neighbour ranks through the comm windows
+  const uint64_t* halo_in_l;  // my window: rank g-1's right edge (read by my block 0)
+  const uint64_t* halo_in_r;  // my window: rank g+1's left edge (read by my last block)
+  uint64_t* halo_out_l;       // rank g-1's window: my left edge (peer pointer)
+  uint64_t* halo_out_r;       // rank g+1's window: my right edge (peer pointer)
 };
 
 // Launch entry points (one per category family).  Return cudaError_t of the launch.

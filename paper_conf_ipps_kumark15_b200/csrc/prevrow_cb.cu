@@ -16,7 +16,12 @@
 //    published edges: case-2 two-way halo of Table II [L265-L274], ([L193-L195]), one exchange
 //    per HB rows instead of one per row.
 //  * Edge exchange = (value, tag) 64-bit pairs in global memory (single-copy atomic): the
-//    consumer polls the data itself, no flag, no fence.  Tag = (fill epoch mod 4096) << 20 | band + 1.
+//    consumer polls the data itself, no flag, no fence.  Tag = (fill epoch mod 2048) << 20 | band + 1
+//    (bit 31 set for multi-GPU fills, whose epoch is the rank-consistent fill count).
+//  * Multi-GPU (lddp_fill_multi): each rank owns a block-aligned column strip; the strip's outer
+//    blocks also push their edges into the neighbour ranks' comm windows (system-scope stores over
+//    NVLink) and take their halos from their own window -- the same two-way exchange, one band
+//    at a time, across GPUs (Table II case 2 [L265-L274], [L193-L195]).
 //  * Cost rows (the HBM stream, 4 B/cell) flow through a per-warp D-row shared-memory ring
 //    filled by 16-byte cp.async (LDGSTS.128, L1 bypass; 8-byte when VP % 4 != 0), D-1 rows ahead
 //    of the row being computed; every lane copies exactly the columns it later reads, so the ring
@@ -122,6 +127,13 @@ __device__ __forceinline__ void cb_st_pair2(uint64_t* p, uint64_t a, uint64_t b)
 __device__ __forceinline__ void cb_ld_pair2(const uint64_t* p, uint64_t& a, uint64_t& b) {
   asm volatile("ld.relaxed.gpu.global.v2.u64 {%0, %1}, [%2];" : "=l"(a), "=l"(b) : "l"(p) : "memory");
 }
+// system scope: edge pairs exchanged with the neighbour GPUs' windows (NVLink peer memory)
+__device__ __forceinline__ void cb_st_pair2_sys(uint64_t* p, uint64_t a, uint64_t b) {
+  asm volatile("st.relaxed.sys.global.v2.u64 [%0], {%1, %2};" ::"l"(p), "l"(a), "l"(b) : "memory");
+}
+__device__ __forceinline__ void cb_ld_pair2_sys(const uint64_t* p, uint64_t& a, uint64_t& b) {
+  asm volatile("ld.relaxed.sys.global.v2.u64 {%0, %1}, [%2];" : "=l"(a), "=l"(b) : "l"(p) : "memory");
+}
 
 // One band of nr <= HB rows.  OUT: this lane holds out-of-table columns (their value is f's
 // boundary value in every row: one extra select per cell, taken only by the two edge blocks'
@@ -204,7 +216,7 @@ __device__ __forceinline__ void cb_band(CbBulk& bk, const CUtensorMap* tmap, con
       T UR = (v < VP - 1) ? cur[v + 1] : rv;
       if (OUT && (VP % 4 != 0 || (v & 3) == 3)) UR = (rfix == v) ? outv[VP - 1] : UR;
       typename F::OutT o;
-      T x = F::f(U, UL, U, UR, typename F::RowCtx(0), typename F::ColCtx(0), g[v], row, e0 + v, p.param_c, o);
+      T x = F::f(U, UL, U, UR, typename F::RowCtx(0), typename F::ColCtx(0), g[v], row, p.col0 + e0 + v, p.param_c, o);
       nw_[v] = x;
       if (TABLE) {
         const int col = e0 + v;
@@ -249,18 +261,21 @@ __global__ void __launch_bounds__(256) prevrow_cb_kernel(const FillParams p, con
     const int j0 = q * BW;
     const int e0 = j0 - HB + lane * VP;   // first column of this lane
     const G* cost = static_cast<const G*>(p.grid);
+    // the table's columns in local coordinates: [clo, chi) (multi-GPU: this rank's strip is
+    // [0, W) of the whole table [-col0, cols_total - col0); its halos reach into the neighbours')
+    const int clo = -p.col0, chi = p.cols_total - p.col0;
     // out-of-table columns keep the boundary value of f in every row
     uint32_t omask = 0;
     T outv[VP];
 #pragma unroll
     for (int v = 0; v < VP; ++v) {
       const int col = e0 + v;
-      if (col < 0 || col >= W) omask |= 1u << v;
-      outv[v] = col < 0 ? F::left(p, 0) : F::right(p, 0);
+      if (col < clo || col >= chi) omask |= 1u << v;
+      outv[v] = col < clo ? F::left(p, 0) : F::right(p, 0);
     }
     const bool anyout = __any_sync(0xffffffffu, omask != 0);
-    const bool lfix = (e0 == 0);                                         // column 0 at v = 0
-    const int rfix = (W - 1 >= e0 && W - 1 < e0 + VP) ? (W - 1 - e0) : -1;   // column W-1
+    const bool lfix = (e0 == clo);                                             // column 0 at v = 0
+    const int rfix = (chi - 1 >= e0 && chi - 1 < e0 + VP) ? (chi - 1 - e0) : -1;   // column W-1
     T eoutv[VP];
 #pragma unroll
     for (int v = 0; v < VP; ++v) eoutv[v] = (v == 0) ? F::left(p, 0) : F::right(p, 0);
@@ -271,7 +286,7 @@ __global__ void __launch_bounds__(256) prevrow_cb_kernel(const FillParams p, con
 #pragma unroll
     for (int s = 0; s < kCbNSeg<VP>; ++s) {
       const int col = e0 + SEG * s;
-      const bool in = col >= 0 && col < W;
+      const bool in = col >= clo && col < chi;
       ssz[s] = in ? 4u * SEG : 0u;
       asm volatile("mov.b32 %0, %0;" : "+r"(ssz[s]));   // opaque: no per-row rematerialisation
       src[s] = cost + (in ? col : 0);
@@ -342,11 +357,13 @@ __global__ void __launch_bounds__(256) prevrow_cb_kernel(const FillParams p, con
     // row -1 (virtual): f's top initialisation
     T cur[VP];
 #pragma unroll
-    for (int v = 0; v < VP; ++v) cur[v] = ((omask >> v) & 1u) ? outv[v] : F::top(p, e0 + v);
+    for (int v = 0; v < VP; ++v) cur[v] = ((omask >> v) & 1u) ? outv[v] : F::top(p, p.col0 + e0 + v);   // global column
 
-    // edge-pair tags: fill epoch (mod 4096) and band + 1 in disjoint bit fields -- every slot a fill
-  // uses is rewritten by it, so a pair left by an earlier fill of this workspace never matches
-  const uint32_t tag0 = (uint32_t)(p.epoch & 0xFFFu) << 20;
+    // edge-pair tags: fill epoch (mod 2048) and band + 1 in disjoint bit fields -- every slot a fill
+    // uses is rewritten by it, so a pair left by an earlier fill of this workspace never matches
+  // (multi-GPU: the rank-consistent fill epoch, with bit 31 set, so the neighbours agree)
+  const bool xrank = p.halo_in_l != nullptr || p.halo_in_r != nullptr;
+  const uint32_t tag0 = xrank ? (0x80000000u | (uint32_t)(p.wepoch & 0x7FFu) << 20) : (uint32_t)(p.epoch & 0x7FFu) << 20;
     uint64_t* edges = reinterpret_cast<uint64_t*>(p.bnd);   // [nb][4 slots][2 sides][HB] pairs
     const bool lhalo = lane < HL, rhalo = lane >= 32 - HL;
     const bool ledge = lane >= HL && lane < 2 * HL;          // own columns [j0, j0 + HB)
@@ -371,22 +388,41 @@ __global__ void __launch_bounds__(256) prevrow_cb_kernel(const FillParams p, con
       const int band = (int)(r0 / HB);
       const uint32_t tag = tag0 | (((uint32_t)band + 1u) & 0xFFFFFu);
       uint64_t* mine = edges + ((size_t)q * 4 + (band & 3)) * 2 * HB;
+      const int xslot = ((int)(p.wepoch & 1) * 4 + (band & 3)) * HB;   // multi-GPU window slot
       if (ledge || redge) {
         uint64_t* d = mine + (ledge ? 0 : HB) + (ledge ? (lane - HL) : (lane - (32 - 2 * HL))) * VP;
 #pragma unroll
         for (int v = 0; v < VP; v += 2)
           cb_st_pair2(d + v, ((uint64_t)tag << 32) | (uint32_t)cur[v], ((uint64_t)tag << 32) | (uint32_t)cur[v + 1]);
+        // multi-GPU: the strip's outer edges also go into the neighbour ranks' windows
+        uint64_t* xo = nullptr;
+        // (8 slots: fill parity x band mod 4 -- a rank may start fill k+1 while its neighbour still
+        // reads fill k's last edges)
+        if (ledge && q == 0 && p.halo_out_l != nullptr) xo = p.halo_out_l + xslot + (lane - HL) * VP;
+        if (redge && q == nb - 1 && p.halo_out_r != nullptr) xo = p.halo_out_r + xslot + (lane - (32 - 2 * HL)) * VP;
+        if (xo != nullptr) {
+#pragma unroll
+          for (int v = 0; v < VP; v += 2)
+            cb_st_pair2_sys(xo + v, ((uint64_t)tag << 32) | (uint32_t)cur[v], ((uint64_t)tag << 32) | (uint32_t)cur[v + 1]);
+        }
       }
       const int nbq = lhalo ? q - 1 : q + 1;
-      const bool need = (lhalo && q > 0) || (rhalo && q + 1 < nb);
+      // halo from the neighbour block of this GPU, or (strip edges) from the neighbour rank
+      const bool xin = (lhalo && q == 0 && p.halo_in_l != nullptr) || (rhalo && q == nb - 1 && p.halo_in_r != nullptr);
+      const bool need = (lhalo && q > 0) || (rhalo && q + 1 < nb) || xin;
       const uint64_t* s = nullptr;
-      if (need)
+      if (xin)
+        s = lhalo ? p.halo_in_l + xslot + lane * VP : p.halo_in_r + xslot + (lane - (32 - HL)) * VP;
+      else if (need)
         s = edges + ((size_t)nbq * 4 + (band & 3)) * 2 * HB + (lhalo ? HB + lane * VP : (lane - (32 - HL)) * VP);
       uint64_t pr[VP];
       bool ok = true;
       if (need) {
 #pragma unroll
-        for (int v = 0; v < VP; v += 2) cb_ld_pair2(s + v, pr[v], pr[v + 1]);
+        for (int v = 0; v < VP; v += 2) {
+          if (xin) cb_ld_pair2_sys(s + v, pr[v], pr[v + 1]);
+          else cb_ld_pair2(s + v, pr[v], pr[v + 1]);
+        }
 #pragma unroll
         for (int v = 0; v < VP; ++v) ok = ok && ((uint32_t)(pr[v] >> 32) == tag);
       }
@@ -397,7 +433,10 @@ __global__ void __launch_bounds__(256) prevrow_cb_kernel(const FillParams p, con
           if (!ok) {
             ok = true;
 #pragma unroll
-            for (int v = 0; v < VP; v += 2) cb_ld_pair2(s + v, pr[v], pr[v + 1]);
+            for (int v = 0; v < VP; v += 2) {
+              if (xin) cb_ld_pair2_sys(s + v, pr[v], pr[v + 1]);
+              else cb_ld_pair2(s + v, pr[v], pr[v + 1]);
+            }
 #pragma unroll
             for (int v = 0; v < VP; ++v) ok = ok && ((uint32_t)(pr[v] >> 32) == tag);
           }
@@ -551,7 +590,7 @@ __global__ void __launch_bounds__(256) prevrow_gh_kernel(const FillParams p, con
 
   // edge-pair tags: fill epoch (mod 4096) and band + 1 in disjoint bit fields -- every slot a fill
   // uses is rewritten by it, so a pair left by an earlier fill of this workspace never matches
-  const uint32_t tag0 = (uint32_t)(p.epoch & 0xFFFu) << 20;
+  const uint32_t tag0 = (uint32_t)(p.epoch & 0x7FFu) << 20;
   uint64_t* edges = reinterpret_cast<uint64_t*>(p.bnd);
   const bool lhalo = lane < HL, rhalo = lane >= 32 - HL;
   const bool ledge = lane >= HL && lane < 2 * HL;

@@ -84,6 +84,8 @@ _SIGS = {
     "lddp_comm_handle": (ctypes.c_int, [_P, ctypes.c_char_p]),
     "lddp_comm_connect": (ctypes.c_int, [_P, ctypes.c_char_p, ctypes.c_char_p]),
     "lddp_comm_connect_local": (ctypes.c_int, [_P, _P, _P]),
+    "lddp_plan_partition": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.c_int32,
+                                           ctypes.POINTER(ctypes.c_int64), ctypes.POINTER(ctypes.c_int64)]),
     "lddp_multi_partition": (ctypes.c_int, [ctypes.c_int64, ctypes.c_int32, ctypes.c_int32,
                                             ctypes.POINTER(ctypes.c_int64), ctypes.POINTER(ctypes.c_int64)]),
     "lddp_comm_destroy": (ctypes.c_int, [_P]),
@@ -199,6 +201,13 @@ def lddp_multi_partition(cols: int, nranks: int, rank: int):
     _check(_lib.lddp_multi_partition(cols, nranks, rank, ctypes.byref(c0), ctypes.byref(c1)),
            "lddp_multi_partition")
     return c0.value, c1.value
+
+
+def lddp_plan_partition(plan, nranks: int, rank: int):
+    lo, hi = ctypes.c_int64(), ctypes.c_int64()
+    _check(_lib.lddp_plan_partition(plan, nranks, rank, ctypes.byref(lo), ctypes.byref(hi)),
+           "lddp_plan_partition")
+    return lo.value, hi.value
 
 
 def lddp_comm_destroy(comm) -> None:

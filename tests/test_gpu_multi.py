@@ -226,3 +226,121 @@ def test_inverted_l_diagonal_shares(func, cat, P, shape):
     finally:
         for c in comms:
             lddp.lddp_comm_destroy(c)
+
+
+# --------------------------------------------------- prev-row column strips, two-way halos
+@pytest.mark.parametrize("func", ["minpath3", "min2plus"])
+@pytest.mark.parametrize("P", [2, 3, 4])
+@pytest.mark.parametrize("shape", [(300, 1024), (1000, 2048), (517, 1540), (64, 4096)])
+def test_prev_row_two_way_halos(func, P, shape):
+    """Previous-row category across P ranks (loopback: all ranks on this GPU, each with its own
+    window, workspace and stream): block-aligned column strips; every band the strips' outer
+    blocks exchange their HB-column edges with the neighbour ranks both ways (Table II case 2,
+    [L193-L195], [L265-L274]).  Several fills with different grids, enqueued rank by rank.  The
+    score is per rank (the minimum of its columns); its minimum over ranks is the oracle's."""
+    import torch
+
+    from paper_conf_ipps_kumark15_b200 import lddp
+    H, W = shape
+    dev = torch.device("cuda:0")
+    plan = lddp.Plan(func, "prev_row", H, W, lddp.OUT_SCORE | lddp.OUT_LAST_ROW | lddp.OUT_TABLE)
+    comms = [lddp.lddp_comm_create(plan.handle, P, r) for r in range(P)]
+    for r in range(P):
+        lddp.lddp_comm_connect_local(comms[r], comms[r + 1] if r + 1 < P else None, comms[r - 1] if r > 0 else None)
+    grids = [(inputs.gen_costs if func == "minpath3" else inputs.gen_init)(17 * k + P + H, H, W) for k in range(3)]
+    tg = [torch.from_numpy(g).to(dev) for g in grids]
+    outs = [(torch.full((P,), -7, dtype=torch.int32, device=dev), torch.full((W,), -7, dtype=torch.int32, device=dev),
+             torch.full((H, W), -7, dtype=torch.int32, device=dev)) for _ in grids]
+    wss = [torch.zeros(plan.ws_bytes, dtype=torch.uint8, device=dev) for _ in range(P)]
+    streams = [torch.cuda.Stream(dev) for _ in range(P)]
+    torch.cuda.synchronize()
+    try:
+        for r in range(P):
+            for g, (sc, lr, tab) in zip(tg, outs):
+                inp, out = plan.io(grid=g, score=sc[r:r + 1], last_row=lr, table=tab)
+                lddp.lddp_fill_multi(plan.handle, inp, out, wss[r].data_ptr(), comms[r], streams[r].cuda_stream)
+        for r in range(P):
+            lddp.lddp_status_check(plan.handle, wss[r].data_ptr(), streams[r].cuda_stream)
+        torch.cuda.synchronize()
+        for g, (sc, lr, tab) in zip(grids, outs):
+            ref = (oracle.minpath3(g, table=True) if func == "minpath3" else oracle.min2plus(g, 1, table=True))
+            np.testing.assert_array_equal(tab.cpu().numpy(), ref.table)
+            np.testing.assert_array_equal(lr.cpu().numpy(), ref.last_row)
+            s = sc.cpu().numpy()
+            for r in range(P):
+                c0, c1 = lddp.lddp_plan_partition(plan.handle, P, r)
+                assert c0 % 4 == 0 and (c1 == W or c1 % 4 == 0)
+                if c1 > c0:
+                    assert s[r] == ref.last_row[c0:c1].min()
+            assert s[s != -7].min() == ref.score
+    finally:
+        for c in comms:
+            lddp.lddp_comm_destroy(c)
+
+
+def _ipc_rank_rows(rank, world, port, func, m, n, fills, q):
+    """One process per rank (all on cuda:0): prev-row column strips through CUDA IPC windows."""
+    import torch
+    import torch.distributed as dist
+
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    from paper_conf_ipps_kumark15_b200 import inputs as inp_mod
+    from paper_conf_ipps_kumark15_b200 import lddp
+    dev = torch.device("cuda:0")
+    torch.cuda.set_device(dev)
+    plan = lddp.Plan(func, "prev_row", m, n, lddp.OUT_SCORE | lddp.OUT_LAST_ROW)
+    comm = lddp.lddp_comm_create(plan.handle, world, rank)
+    handles = [None] * world
+    dist.all_gather_object(handles, lddp.lddp_comm_handle(comm))
+    lddp.lddp_comm_connect(comm, handles[rank + 1] if rank + 1 < world else None,
+                           handles[rank - 1] if rank > 0 else None)
+    dist.barrier()
+    c0, c1 = lddp.lddp_plan_partition(plan.handle, world, rank)
+    stream = torch.cuda.current_stream(dev)
+    if rank == 1:
+        time.sleep(0.5)   # rank 0's kernel waits at its first band exchange
+    bufs = []
+    gen = inp_mod.gen_costs if func == "minpath3" else inp_mod.gen_init
+    for k in range(fills):
+        g = torch.from_numpy(gen(2000 + 17 * k, m, n)).to(dev)
+        sc = torch.full((1,), -7, dtype=torch.int32, device=dev)
+        lr = torch.full((n,), -7, dtype=torch.int32, device=dev)
+        inp, out = plan.io(grid=g, score=sc, last_row=lr)
+        lddp.lddp_fill_multi(plan.handle, inp, out, plan.ws.data_ptr(), comm, stream.cuda_stream)
+        bufs.append((g, sc, lr))
+    lddp.lddp_status_check(plan.handle, plan.ws.data_ptr(), stream.cuda_stream)
+    res = [(int(sc.cpu().numpy()[0]), lr.cpu().numpy()[c0:c1].tolist()) for g, sc, lr in bufs]
+    dist.barrier()
+    lddp.lddp_comm_destroy(comm)
+    q.put((rank, c0, c1, res))
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("func,world", [("minpath3", 2), ("minpath3", 3), ("min2plus", 2)])
+def test_cross_process_ipc_prev_row(func, world):
+    """Prev-row two-way halos between PROCESSES (CUDA IPC windows, handles over gloo), three
+    back-to-back fills with different grids; strips from lddp_plan_partition tile [0, n)."""
+    import torch.multiprocessing as mp
+    m, n, fills = 700, 1536, 3
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_ipc_rank_rows, args=(r, world, port, func, m, n, fills, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    parts = sorted([q.get(timeout=300) for _ in range(world)])
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    assert parts[0][1] == 0 and parts[-1][2] == n
+    assert all(parts[i][2] == parts[i + 1][1] for i in range(world - 1))
+    for k in range(fills):
+        g = (inputs.gen_costs if func == "minpath3" else inputs.gen_init)(2000 + 17 * k, m, n)
+        ref = oracle.minpath3(g) if func == "minpath3" else oracle.min2plus(g, 1)
+        last = np.zeros(n, np.int32)
+        for rank, c0, c1, res in parts:
+            last[c0:c1] = res[k][1]
+            assert res[k][0] == (last[c0:c1].min() if c1 > c0 else -7)
+        np.testing.assert_array_equal(last, ref.last_row)
+        assert min(r[3][k][0] for r in parts if r[2] > r[1]) == ref.score

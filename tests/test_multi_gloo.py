@@ -114,3 +114,86 @@ def test_library_partition():
             assert min(sizes) >= 1 and max(sizes) - min(sizes) <= 1
     with pytest.raises(lddp.LddpError):
         lddp.lddp_multi_partition(10, 2, 2)
+
+
+# ------------------------------------------------- prev-row: two-way trapezoid halos over gloo
+HB = 32          # band height = halo width of the column-block kernel's default geometry
+BW = 64          # its own columns per block: strips are whole blocks
+GARBAGE = -(1 << 40)   # value of a halo cell whose inputs are stale (must never reach own columns)
+
+
+def _rows_rank_main(rank, world, port, m, n, seed, q):
+    """Rank g owns whole BW-column blocks; every band of HB rows it computes its columns plus HB
+    halo columns each side from the halo values exchanged at the band start (one send + one recv
+    per side and band: Table II case 2 two-way halo [L265-L274], [L193-L195]).  Cells are the
+    min-path recurrence c + min(UL, U, UR) [L298]; a halo cell whose left / right input lies
+    outside the extended window takes GARBAGE, so a too-narrow halo would corrupt own columns."""
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    from paper_conf_ipps_kumark15_b200 import inputs
+    cost = inputs.gen_costs(seed, m, n).astype(np.int64)
+    NB = (n + BW - 1) // BW
+    c0 = min(rank * NB // world * BW, n)
+    c1 = min((rank + 1) * NB // world * BW, n)
+    big = np.int64(1 << 50)                       # out-of-table neighbour (f's boundary)
+    lo, hi = c0 - HB, c1 + HB                     # extended window [lo, hi)
+    cols = np.arange(lo, hi)
+    inside = (cols >= 0) & (cols < n)
+    cur = np.where(inside, 0, big).astype(np.int64)   # row -1: top initialisation
+    for r0 in range(0, m, HB):
+        nr = min(HB, m - r0)
+        for i in range(r0, r0 + nr):
+            ul = np.concatenate([[GARBAGE], cur[:-1]])
+            ur = np.concatenate([cur[1:], [GARBAGE]])
+            ul[0] = big if lo - 1 < 0 else GARBAGE
+            ur[-1] = big if hi >= n else GARBAGE
+            c = np.where(inside, cost[i, np.clip(cols, 0, n - 1)], 0)
+            nxt = c + np.minimum(np.minimum(ul, cur), ur)
+            cur = np.where(inside, nxt, big)
+        if r0 + HB >= m:
+            break
+        # band boundary: own edges out, neighbours' edges in (both directions)
+        reqs = []
+        if rank > 0:
+            reqs.append(dist.isend(torch.from_numpy(cur[HB:2 * HB].copy()), dst=rank - 1))
+        if rank + 1 < world:
+            reqs.append(dist.isend(torch.from_numpy(cur[-2 * HB:-HB].copy()), dst=rank + 1))
+        if rank > 0:
+            t = torch.zeros(HB, dtype=torch.int64)
+            dist.recv(t, src=rank - 1)
+            cur[:HB] = t.numpy()
+        if rank + 1 < world:
+            t = torch.zeros(HB, dtype=torch.int64)
+            dist.recv(t, src=rank + 1)
+            cur[-HB:] = t.numpy()
+        for rq in reqs:
+            rq.wait()
+    own = cur[HB:HB + (c1 - c0)]
+    q.put((rank, c0, c1, own.tolist()))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_prev_row_two_way_halo_gloo(world):
+    import oracle
+    from paper_conf_ipps_kumark15_b200 import inputs
+    m, n, seed = 301, 448, 9
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_rows_rank_main, args=(r, world, port, m, n, seed, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    parts = sorted(q.get(timeout=240) for _ in range(world))
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    assert parts[0][1] == 0 and parts[-1][2] == n
+    last = np.zeros(n, np.int64)
+    for rank, c0, c1, row in parts:
+        assert c0 % BW == 0
+        last[c0:c1] = row
+    ref = oracle.minpath3(inputs.gen_costs(seed, m, n))
+    np.testing.assert_array_equal(last, ref.last_row)
+    assert last.min() == ref.score
