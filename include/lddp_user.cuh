@@ -201,6 +201,8 @@ inline lddp_status fill(const Problem& pb, void* workspace, cudaStream_t stream)
   p.timeout_ns = 30ull * 1000000000ull;
   p.one = 1;
   p.spin_polls = 256;
+  p.diag_lo = -(pb.rows - 1);   // inverted-L: every diagonal d = j - i
+  p.diag_hi = pb.cols;
   cudaError_t e = cudaSuccess;
   const bool tab = pb.table != nullptr;
   // check() guarantees the category orders kMask, so only the kernels whose schedule can run

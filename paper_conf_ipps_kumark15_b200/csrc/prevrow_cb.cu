@@ -135,6 +135,22 @@ __device__ __forceinline__ void cb_ld_pair2_sys(const uint64_t* p, uint64_t& a, 
   asm volatile("ld.relaxed.sys.global.v2.u64 {%0, %1}, [%2];" : "=l"(a), "=l"(b) : "l"(p) : "memory");
 }
 
+// Table-edge masks of an edge warp (see cb_band): lv' = (lv & lA) | lO, UR'[v] = (UR & rA[v]) | rO[v]
+template <int VP>
+struct CbEdge {
+  uint32_t lA, lO;
+  uint32_t rA[VP], rO[VP];
+};
+template <class T>
+__device__ __forceinline__ T cb_fix(T x, uint32_t A, uint32_t O) {
+  static_assert(sizeof(T) == 4, "32-bit cells");
+  uint32_t u;
+  memcpy(&u, &x, 4);
+  u = (u & A) | O;
+  memcpy(&x, &u, 4);
+  return x;
+}
+
 // One band of nr <= HB rows.  OUT: this lane holds out-of-table columns (their value is f's
 // boundary value in every row: one extra select per cell, taken only by the two edge blocks'
 // edge lanes -- warp-uniform for every other warp).
@@ -144,8 +160,7 @@ __device__ __forceinline__ void cb_band(CbBulk& bk, const CUtensorMap* tmap, con
                                         const typename F::GridT* ring, int& cslot, uint32_t& idst, int& ileft,
                                         int64_t& ioff, const int64_t pitch,
                                         const typename F::GridT* const (&src)[kCbNSeg<VP>], const uint32_t (&ssz)[kCbNSeg<VP>],
-                                        const typename F::T (&outv)[VP], const uint32_t omask, const bool lfix,
-                                        const int rfix, const int e0,
+                                        const CbEdge<VP>& ed, const int e0,
                                         const int j0, const int BW) {
   using T = typename F::T;
   using G = typename F::GridT;
@@ -207,14 +222,18 @@ __device__ __forceinline__ void cb_band(CbBulk& bk, const CUtensorMap* tmap, con
     // e0 % 4 == 0) and column W-1's UR (v % 4 == 3 since W % 4 == 0).  Forcing every outside
     // cell every row put selects on the row chain and made the two edge warps -- which pace all
     // others through the halo exchange -- twice as slow as an interior warp.
-    if (OUT && lfix) lv = outv[0];
+    // The fix is one LOP3 per edge cell, (x & A) | O with per-lane masks set once (A = 0, O =
+    // the boundary value's bits on the lane holding the table edge; A = ~0, O = 0 elsewhere):
+    // selects here let the compiler serialise the two shuffles of a row pair behind them (C4
+    // edge warps 108 vs 64 cycles per row, pacing every warp through the exchange).
+    if (OUT) lv = cb_fix(lv, ed.lA, ed.lO);
     T nw_[VP];
 #pragma unroll
     for (int v = 0; v < VP; ++v) {
       const T UL = (v > 0) ? cur[v - 1] : lv;
       const T U = cur[v];
       T UR = (v < VP - 1) ? cur[v + 1] : rv;
-      if (OUT && (VP % 4 != 0 || (v & 3) == 3)) UR = (rfix == v) ? outv[VP - 1] : UR;
+      if (OUT && (VP % 4 != 0 || (v & 3) == 3)) UR = cb_fix(UR, ed.rA[v], ed.rO[v]);
       typename F::OutT o;
       T x = F::f(U, UL, U, UR, typename F::RowCtx(0), typename F::ColCtx(0), g[v], row, p.col0 + e0 + v, p.param_c, o);
       nw_[v] = x;
@@ -273,12 +292,29 @@ __global__ void __launch_bounds__(256) prevrow_cb_kernel(const FillParams p, con
       if (col < clo || col >= chi) omask |= 1u << v;
       outv[v] = col < clo ? F::left(p, 0) : F::right(p, 0);
     }
-    const bool anyout = __any_sync(0xffffffffu, omask != 0);
+    bool anyout = __any_sync(0xffffffffu, omask != 0);
+    if (p.debug & 16) anyout = false;   // development timing switches (wrong edge results)
+    if (p.debug & 32) anyout = true;
     const bool lfix = (e0 == clo);                                             // column 0 at v = 0
     const int rfix = (chi - 1 >= e0 && chi - 1 < e0 + VP) ? (chi - 1 - e0) : -1;   // column W-1
-    T eoutv[VP];
+    CbEdge<VP> ed;
+    {
+      const T lb = F::left(p, 0), rb = F::right(p, 0);
+      uint32_t lbits, rbits;
+      memcpy(&lbits, &lb, 4);
+      memcpy(&rbits, &rb, 4);
+      ed.lA = lfix ? 0u : ~0u;
+      ed.lO = lfix ? lbits : 0u;
 #pragma unroll
-    for (int v = 0; v < VP; ++v) eoutv[v] = (v == 0) ? F::left(p, 0) : F::right(p, 0);
+      for (int v = 0; v < VP; ++v) {
+        ed.rA[v] = (rfix == v) ? 0u : ~0u;
+        ed.rO[v] = (rfix == v) ? rbits : 0u;
+        asm volatile("mov.b32 %0, %0;" : "+r"(ed.rA[v]));   // opaque: kept as LOP3 masks
+        asm volatile("mov.b32 %0, %0;" : "+r"(ed.rO[v]));
+      }
+      asm volatile("mov.b32 %0, %0;" : "+r"(ed.lA));
+      asm volatile("mov.b32 %0, %0;" : "+r"(ed.lO));
+    }
     // 16-byte segments of this lane: all in or all out (W % 4 == 0, e0 % 4 == 0)
     constexpr int SEG = kCbSeg<VP>;
     uint32_t ssz[kCbNSeg<VP>];
@@ -376,9 +412,9 @@ __global__ void __launch_bounds__(256) prevrow_cb_kernel(const FillParams p, con
       const bool trc = p.trace != nullptr && q == p.trace_chunks && lane == 0 && r0 / HB < 4096;
       const long long tb0 = trc ? clock64() : 0;
       if (anyout)
-        cb_band<F, VP, D, TABLE, true, MODE>(bk, tmap, lane, p, cur, g, nr, r0, ring, cslot, idst, ileft, ioff, pitch, src, ssz, eoutv, omask, lfix, rfix, e0, j0, BW);
+        cb_band<F, VP, D, TABLE, true, MODE>(bk, tmap, lane, p, cur, g, nr, r0, ring, cslot, idst, ileft, ioff, pitch, src, ssz, ed, e0, j0, BW);
       else
-        cb_band<F, VP, D, TABLE, false, MODE>(bk, tmap, lane, p, cur, g, nr, r0, ring, cslot, idst, ileft, ioff, pitch, src, ssz, eoutv, omask, lfix, rfix, e0, j0, BW);
+        cb_band<F, VP, D, TABLE, false, MODE>(bk, tmap, lane, p, cur, g, nr, r0, ring, cslot, idst, ileft, ioff, pitch, src, ssz, ed, e0, j0, BW);
       if (trc) {
         p.trace[2 * (r0 / HB)] = (uint64_t)(clock64() - tb0);
       }
