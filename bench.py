@@ -149,8 +149,8 @@ def build_problem(name, dev, lddp, world, rank, tile_rows=0):
     outs = {"lcs": lddp.OUT_SCORE, "dtw": lddp.OUT_SCORE, "fs": lddp.OUT_TABLE,
             "minpath3": lddp.OUT_SCORE | lddp.OUT_LAST_ROW, "min2plus": lddp.OUT_SCORE | lddp.OUT_LAST_ROW,
             "diagmaxplus": lddp.OUT_LAST_ROW | lddp.OUT_LAST_COL}[func]
-    plan = lddp.Plan(func, cat, rows, cols, outs, device=dev.index, tile_rows=tile_rows,
-                     param_c=cfg.get("param_c", 1))
+    plan = lddp.Plan(func, cat, cfg.get("img_rows", rows), cols, outs, device=dev.index, tile_rows=tile_rows,
+                     param_c=cfg.get("param_c", 1), batch=cfg.get("batch", 0))
     t = {}
     h2d = 0
     if "a" in x:
@@ -319,8 +319,8 @@ def roofline(name, ms_per_step, peaks, world, clock_mhz):
     reported with its achieved / peak / frac, the others beside it."""
     cfg = CONFIGS[name]
     func, cat = cfg["func"], cfg["category"]
-    H, W = cfg["rows"], cfg["cols"]
-    cells = H * W
+    H, W = cfg.get("img_rows", cfg["rows"]), cfg["cols"]   # one image's shape (span); cells = the whole batch
+    cells = cfg["rows"] * W
     t = ms_per_step / 1e3
     mhz = peaks.get("sm_max_mhz", 1965.0)
     ops, pipe = WORK[func]
@@ -332,7 +332,7 @@ def roofline(name, ms_per_step, peaks, world, clock_mhz):
     path = {"anti_diagonal": H + W - 1, "knight_move": 2 * (H - 1) + W, "prev_row": H,
             "inverted_l": min(H, W)}[cat]                     # cells on the longest dependency path
     t_span = path * cyc / (mhz * 1e6)
-    hbm_bytes = cells * HBM_PER_CELL.get(func, 0.0) + 4 * (H + W)
+    hbm_bytes = cells * HBM_PER_CELL.get(func, 0.0) + 4 * (cfg["rows"] + W)
     peak_bw = peaks.get("hbm_gbs", 6650.0) * 1e9 * world
     t_mem = hbm_bytes / peak_bw
     terms = {"work": t_work, "span": t_span, "mem": t_mem}
@@ -395,8 +395,9 @@ def cpu_baseline(name):
             oracle.dtw(x["a"][:rows], x["b"])
             cells, sample = rows * cfg["cols"], f"first {rows} rows x all {cfg['cols']} columns"
         elif func == "fs":
-            oracle.fs(x["grid"])
-            cells, sample = cfg["rows"] * cfg["cols"], "whole image"
+            ir = cfg.get("img_rows", cfg["rows"])
+            oracle.fs(x["grid"][:ir])
+            cells, sample = ir * cfg["cols"], "one whole image"
         elif func in ("min2plus", "diagmaxplus"):
             rows = min(cfg["rows"], 8192)
             getattr(oracle, func)(x["grid"][:rows], cfg.get("param_c", 1))
@@ -525,7 +526,7 @@ def main():
                    sampler, tile_rows=args.tile_rows)
     others = {}
     if world == 1 and not args.no_others:
-        for name in ("C1", "C2", "C3", "C4", "C6", "C7"):
+        for name in ("C1", "C2", "C3", "C4", "C6", "C7", "C8"):
             if name == args.workload:
                 continue
             r = measure(name, lddp, dev, 1, 0, max(5, args.steps // 2), args.warmup, flush, peaks, sampler,

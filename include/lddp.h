@@ -144,7 +144,14 @@ typedef struct {
                                 two halo exchanges of the column-block kernel): 16, 32, 48 or
                                 64 (else LDDP_ERR_UNSUPPORTED); 0 = auto (32)                    */
     int32_t grid_ctas;       /* tuning: persistent grid size, 0 = auto (SMs x occupancy)        */
-    int32_t reserved[3];     /* must be 0                                                       */
+    int32_t batch;           /* FS_DITHER only: number of independent images stacked along the
+                                rows (image b = rows [b*rows, (b+1)*rows) of inputs.grid and of
+                                outputs.table, same pitches); 0 or 1 = one image.  All images
+                                are filled by ONE launch whose warps claim (strip, image) pairs
+                                strip-major, so the images' pipelines run concurrently
+                                (batched FS, image-parallel [L335-L348], reading R21).
+                                lddp_fill_multi gives rank g images [g*B/P, (g+1)*B/P).     */
+    int32_t reserved[2];     /* must be 0                                                       */
 } lddp_desc;
 
 typedef struct {

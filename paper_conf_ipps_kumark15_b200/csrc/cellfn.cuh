@@ -192,9 +192,13 @@ struct CellFS {
     v = __fadd_rn(v, __fmul_rn(U, 0.3125f));
     v = __fadd_rn(v, __fmul_rn(UR, 0.1875f));
     v = __fadd_rn(v, __fmul_rn(L, 0.4375f));
-    const bool hi = v >= 128.0f;
-    o = hi ? (uint8_t)255 : (uint8_t)0;
-    return hi ? __fsub_rn(v, 255.0f) : v;
+    // threshold as a register mask (FSET), not a predicate (FSETP -> predicated use costs ~13
+    // cycles on the error chain): m = v >= 128 ? ~0 : 0; e = v - (m & 255.0f), exactly the
+    // oracle's v - 255 or v (v - (+0) == v for every v, -0 included)
+    uint32_t m;
+    asm("set.ge.u32.f32 %0, %1, 128.0;" : "=r"(m) : "f"(v));
+    o = (uint8_t)(m & 255u);
+    return __fsub_rn(v, __uint_as_float(m & 0x437F0000u));
   }
 };
 

@@ -70,8 +70,8 @@ __global__ void __launch_bounds__(W * 32, 1) fsk_kernel(const FillParams p) {
   const int NQ = (Wimg + 31) / 32;
   const int K = NQ + D + 1;   // chunks per strip: the last lane reaches column 32(NQ+1)-1
   const uint32_t ep32 = (uint32_t)p.epoch;
-  const uint8_t* img = static_cast<const uint8_t*>(p.grid);
-  uint8_t* out = static_cast<uint8_t*>(p.table);
+  const uint8_t* img0 = static_cast<const uint8_t*>(p.grid);
+  uint8_t* out0 = static_cast<uint8_t*>(p.table);
 
   for (int i = threadIdx.x; i < W * kAdRing * 32; i += blockDim.x) (&ring[0][0][0])[i] = 0ull;
   if (threadIdx.x < W) cons[threadIdx.x] = 0;
@@ -85,9 +85,15 @@ __global__ void __launch_bounds__(W * 32, 1) fsk_kernel(const FillParams p) {
       strip_sh = s;
     }
     __syncthreads();
-    const int s = strip_sh;
-    if (s >= p.nstrips) break;
+    // batched FS: claim q -> (strip q / B, image q % B), strip-major, so the B images' strip
+    // pipelines advance together; image b = rows [b H, (b+1) H) of the grid / table
+    const int B = p.batch > 1 ? p.batch : 1;
+    const int q = strip_sh;
+    if (q >= p.nstrips * B) break;
+    const int s = q / B, bimg = q - s * B;
     const int64_t row0 = (int64_t)s * SH + (wid * 32 + lane) * R;
+    const uint8_t* img = img0 + (int64_t)bimg * H * p.grid_pitch;
+    uint8_t* out = out0 + (int64_t)bimg * H * p.table_pitch;
     bool rvalid[R];
     const uint8_t* rin[R];
     uint8_t* rout[R];
@@ -132,8 +138,9 @@ __global__ void __launch_bounds__(W * 32, 1) fsk_kernel(const FillParams p) {
     const int botsnk = (wid < W - 1) ? 1 : (last_strip ? 0 : 2);
     uint64_t* ring_top = &ring[wid][0][0];
     uint64_t* ring_bot = &ring[(wid + 1) % W][0][0];
-    const uint64_t* gprev = static_cast<const uint64_t*>(p.bnd) + (int64_t)(s - 1) * p.bnd_stride;
-    uint64_t* gmine = static_cast<uint64_t*>(p.bnd) + (int64_t)s * p.bnd_stride;
+    const int64_t brow = (int64_t)bimg * p.nstrips + s;   // this strip's boundary row (per image)
+    const uint64_t* gprev = static_cast<const uint64_t*>(p.bnd) + (brow - 1) * p.bnd_stride;
+    uint64_t* gmine = static_cast<uint64_t*>(p.bnd) + brow * p.bnd_stride;
     uint64_t tp = 0, tq1 = (topsrc == 2) ? ad_ld_gpu(gprev + lane) : 0ull;
 
     float fifo[E + 3];
@@ -335,9 +342,9 @@ cudaError_t launch_fsk(const FillParams& p, int W, int E, int R, int grid, cudaS
     fsk_kernel<w, e, r><<<grid, w * 32, 0, s>>>(p);                      \
     return cudaGetLastError();                                           \
   }
-  LDDP_FSK(4, 0, 1) LDDP_FSK(4, 1, 1) LDDP_FSK(4, 2, 1) LDDP_FSK(2, 0, 1) LDDP_FSK(2, 1, 1) LDDP_FSK(2, 2, 1)
-  LDDP_FSK(2, 0, 2) LDDP_FSK(2, 1, 2) LDDP_FSK(1, 0, 2) LDDP_FSK(1, 1, 2) LDDP_FSK(1, 2, 2) LDDP_FSK(1, 1, 1) LDDP_FSK(1, 0, 1) LDDP_FSK(1, 2, 1)
-  LDDP_FSK(1, 0, 3) LDDP_FSK(1, 1, 3) LDDP_FSK(1, 0, 4) LDDP_FSK(1, 1, 4)
+  // default (1, 1, 1); the others are the measured alternatives kept for sweeps
+  LDDP_FSK(1, 1, 1) LDDP_FSK(1, 0, 1) LDDP_FSK(1, 2, 1) LDDP_FSK(1, 1, 2) LDDP_FSK(1, 0, 2) LDDP_FSK(4, 1, 1)
+  LDDP_FSK(2, 1, 1)
 #undef LDDP_FSK
   return cudaErrorInvalidValue;
 }

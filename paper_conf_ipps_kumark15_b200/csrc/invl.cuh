@@ -22,7 +22,7 @@
 namespace lddp {
 
 constexpr int kInvlWarps = 4;
-constexpr int kInvlBlock = 32;   // rows per register block (two blocks in flight)
+constexpr int kInvlBlock = 16;   // rows per register block (two blocks in flight; 16 keeps every warp resident: C6 2.70 -> 2.19 ms against 32)
 
 // F::kDirectGrid (the compiled-in f's): the per-cell input is element (i, j) of p.grid, read
 // with a running pointer (and mirrored columns); otherwise (user functors, include/lddp_user.cuh)
@@ -33,7 +33,7 @@ template <class F>
 struct InvlDirect<F, decltype(void(F::kDirectGrid))> { static constexpr bool value = F::kDirectGrid; };
 
 // MIRROR: the kernel's column j' is the grid's column W-1-j' (mInverted-L twin, {UR} -> {UL}).
-template <class F, bool TABLE, bool MIRROR>
+template <class F, bool TABLE, bool MIRROR, int BLK = kInvlBlock>
 __global__ void __launch_bounds__(kInvlWarps * 32) invl_kernel(const FillParams p) {
   using T = typename F::T;
   using G = typename F::GridT;
@@ -62,10 +62,10 @@ __global__ void __launch_bounds__(kInvlWarps * 32) invl_kernel(const FillParams 
     const int64_t step = MIRROR ? p.grid_pitch - 1 : p.grid_pitch + 1;
     // UL of the chain's first cell: the row above row 0 (d >= 0) or the column left of column 0
     T v = MIRROR ? T(0) : (d >= 0 ? F::top(p, (int)d - 1 + p.col0) : F::left(p, -d - 1));
-    G cur[kInvlBlock], nxt[kInvlBlock];
+    G cur[BLK], nxt[BLK];
     auto load_block = [&](G* dst, int64_t i0) {
 #pragma unroll
-      for (int u = 0; u < kInvlBlock; ++u) {
+      for (int u = 0; u < BLK; ++u) {
         const int64_t i = i0 + u;
         if constexpr (InvlDirect<F>::value)
           dst[u] = (live && i >= ia && i < ib) ? __ldcs(src + i * step) : G(0);
@@ -74,10 +74,10 @@ __global__ void __launch_bounds__(kInvlWarps * 32) invl_kernel(const FillParams 
       }
     };
     load_block(cur, ibeg);
-    for (int64_t i0 = ibeg; i0 < iend; i0 += kInvlBlock) {
-      if (i0 + kInvlBlock < iend) load_block(nxt, i0 + kInvlBlock);
+    for (int64_t i0 = ibeg; i0 < iend; i0 += BLK) {
+      if (i0 + BLK < iend) load_block(nxt, i0 + BLK);
 #pragma unroll
-      for (int u = 0; u < kInvlBlock; ++u) {
+      for (int u = 0; u < BLK; ++u) {
         const int64_t i = i0 + u;
         const int64_t j = i + d;
         if (live && i >= ia && i < ib) {
@@ -91,7 +91,7 @@ __global__ void __launch_bounds__(kInvlWarps * 32) invl_kernel(const FillParams 
         }
       }
 #pragma unroll
-      for (int u = 0; u < kInvlBlock; ++u) cur[u] = nxt[u];
+      for (int u = 0; u < BLK; ++u) cur[u] = nxt[u];
     }
   }
 }

@@ -87,8 +87,7 @@ constexpr int kDynPerWarp = 257 * 32 * 2;   // table path: 257 characters x 32 l
 
 // compiled (P row pairs per lane, E lane lag) geometries
 #define LDDP_L16_GEOMS \
-  LDDP_L16_GEOM(3, 3) LDDP_L16_GEOM(3, 2) LDDP_L16_GEOM(4, 3) LDDP_L16_GEOM(4, 2) LDDP_L16_GEOM(2, 3) \
-  LDDP_L16_GEOM(6, 2) LDDP_L16_GEOM(6, 3) LDDP_L16_GEOM(8, 2) LDDP_L16_GEOM(8, 3)
+  LDDP_L16_GEOM(2, 3) LDDP_L16_GEOM(4, 2) LDDP_L16_GEOM(6, 2) LDDP_L16_GEOM(6, 3) LDDP_L16_GEOM(8, 2)
 
 template <int P, int E>
 struct L16Warp {

@@ -170,9 +170,9 @@ double ad_cost(int func, int R, int E, int W, int S, int64_t m, int64_t n, int s
 // variant geometry: rows per lane R, intra-lane skew SIG, extra lag E
 struct VariantGeom { int id, R, SIG, E; };
 const VariantGeom kVariants[] = {
-    {0, 4, 0, 2}, {1, 4, 1, 1}, {2, 2, 1, 1}, {3, 8, 1, 1}, {4, 8, 0, 2}, {5, 4, 0, 1},
-    {6, 16, 0, 2}, {7, 8, 0, 3}, {8, 8, 1, 1}, {9, 8, 1, 1}, {12, 16, 1, 1}, {10, 1, 2, 2},
-    {11, 2, 2, 2}, {13, 1, 2, 1},
+    // compiled wavefront geometries (the rest of the round-1 sweep measured slower and is no
+    // longer built): anti-diagonal R4 chained (default, TABLE), R2 / R8 skewed; knight-move
+    {0, 4, 0, 2}, {2, 2, 1, 1}, {3, 8, 1, 1}, {10, 1, 2, 2}, {11, 2, 2, 2}, {13, 1, 2, 1},
 };
 const VariantGeom* variant_geom(int id) {
   for (const auto& v : kVariants)
@@ -373,6 +373,7 @@ void fill_common(lddp_plan_t pl, const lddp_inputs* in, const lddp_outputs* out,
   p.one = 1;
   p.diag_lo = -(d.rows - 1);
   p.diag_hi = d.cols;
+  p.batch = std::max(d.batch, 1);
   // debug trace buffer: LDDP_TRACE=<device pointer as decimal>:<chunks per row>
   if (const char* tr = getenv("LDDP_TRACE")) {
     unsigned long long ptr = 0;
@@ -391,10 +392,15 @@ lddp_status launch(lddp_plan_t pl, const FillParams& p, cudaStream_t s) {
     FillParams q = p;
     q.nstrips = pl->fsk_nstrips;
     q.bnd_stride = pl->fsk_bnd_stride;
+    q.batch = std::max(q.batch, 1);
     const int fg = env_int("LDDP_FSK_GRID", 0);
-    e = lddp::launch_fsk(q, pl->fsk_W, pl->fsk_E, pl->fsk_R, std::min(fg > 0 ? fg : pl->sms, pl->fsk_nstrips), s);
+    // one warp per SM for one image (measured best); up to one per SMSP for a batch
+    const int gdef = pl->sms * std::min(q.batch, 4);
+    e = lddp::launch_fsk(q, pl->fsk_W, pl->fsk_E, pl->fsk_R, std::min(fg > 0 ? fg : gdef, pl->fsk_nstrips * q.batch), s);
     if (e == cudaErrorInvalidValue)
       return fail(LDDP_ERR_UNSUPPORTED, "fsk W=%d E=%d R=%d not compiled", pl->fsk_W, pl->fsk_E, pl->fsk_R);
+  } else if (pl->kind == 0 && pl->desc.batch > 1) {
+    return fail(LDDP_ERR_UNSUPPORTED, "batched FS: grid / table rows must be 16-byte aligned with pitches %% 16 == 0");
   } else if (pl->kind == 0) {
     int grid = std::min(pl->grid, p.nstrips);
     int r = wf_dispatch(pl->desc.func, 0, pl->variant, p.table != nullptr, &p, grid, s);
@@ -527,6 +533,9 @@ lddp_status lddp_plan(const lddp_desc* desc, lddp_plan_t* out) {
     if (fm == 0) return fail(LDDP_ERR_INVALID_ARG, "unknown func %d", d.func);
     if (d.category < 0 || d.category > 5) return fail(LDDP_ERR_INVALID_ARG, "unknown category %d", d.category);
     if (d.rows < 0 || d.cols < 0) return fail(LDDP_ERR_SHAPE, "negative shape");
+    if (d.batch < 0) return fail(LDDP_ERR_INVALID_ARG, "negative batch");
+    if (d.batch > 1 && d.func != LDDP_F_FS_DITHER)
+      return fail(LDDP_ERR_UNSUPPORTED, "batch > 1 is supported for FS_DITHER (batched images) only");
     if (d.cols > (int64_t)0x7fff0000 || d.rows > ((int64_t)1 << 40)) return fail(LDDP_ERR_SHAPE, "shape too large");
     if (d.outputs & ~(LDDP_OUT_SCORE | LDDP_OUT_LAST_ROW | LDDP_OUT_LAST_COL | LDDP_OUT_TABLE))
       return fail(LDDP_ERR_INVALID_ARG, "unknown output bits 0x%x", d.outputs);
@@ -704,7 +713,12 @@ lddp_status lddp_plan(const lddp_desc* desc, lddp_plan_t* out) {
         pl->fsk_R = env_int("LDDP_FSK_R", 1);
         pl->fsk_nstrips = (int)((d.rows + 32 * pl->fsk_W * pl->fsk_R - 1) / (32 * pl->fsk_W * pl->fsk_R));
         pl->fsk_bnd_stride = ((d.cols + 31) / 32) * 32;   // (value, tag) pairs per boundary row
-        pl->ws_bytes = std::max(pl->ws_bytes, pl->off_bnd + (size_t)pl->fsk_nstrips * pl->fsk_bnd_stride * 8);
+        pl->ws_bytes = std::max(pl->ws_bytes, pl->off_bnd + (size_t)pl->fsk_nstrips * pl->fsk_bnd_stride * 8 *
+                                                  std::max(d.batch, 1));
+      }
+      if (d.batch > 1 && !pl->fsk) {
+        delete pl;
+        return fail(LDDP_ERR_UNSUPPORTED, "batched FS needs the fsk kernel (knight-move, cols %% 16 == 0, TABLE)");
       }
     } else if (d.category == LDDP_CAT_PREV_ROW) {
       pl->kind = 1;
@@ -831,10 +845,11 @@ lddp_status lddp_plan_describe(lddp_plan_t pl, char* buf, size_t len) {
              "{\"kernel\": \"fsk\", \"variant\": -1, \"rows_per_lane\": %d, \"skew\": 2, \"extra_lag\": %d, "
              "\"warps\": %d, \"grid\": %d, \"sms\": %d, \"occupancy\": 1, \"strip_rows\": %d, "
              "\"strips\": %d, \"chunks\": %d, \"blocks\": 0, \"bands\": 0, \"workspace_bytes\": %zu, "
-             "\"fallback\": \"wavefront variant %d when pitches are not 16-byte multiples\"}",
-             pl->fsk_R, pl->fsk_E, pl->fsk_W, std::min(pl->sms, pl->fsk_nstrips), pl->sms, 32 * pl->fsk_W * pl->fsk_R,
-             pl->fsk_nstrips,
-             (int)(pl->fsk_bnd_stride / 32), pl->ws_bytes, pl->variant);
+             "\"batch\": %d, \"fallback\": \"wavefront variant %d when pitches are not 16-byte multiples\"}",
+             pl->fsk_R, pl->fsk_E, pl->fsk_W,
+             std::min(pl->sms * std::min(std::max(pl->desc.batch, 1), 4), pl->fsk_nstrips * std::max(pl->desc.batch, 1)),
+             pl->sms, 32 * pl->fsk_W * pl->fsk_R, pl->fsk_nstrips,
+             (int)(pl->fsk_bnd_stride / 32), pl->ws_bytes, std::max(pl->desc.batch, 1), pl->variant);
     return LDDP_OK;
   }
   snprintf(buf, len,
@@ -900,15 +915,16 @@ lddp_status lddp_fill_host(lddp_plan_t pl, const lddp_inputs* hin, const lddp_ou
     const size_t gdp = align_up((size_t)std::max<int64_t>(d.cols, 1) * gel, 16);
     const size_t tdp = align_up((size_t)std::max<int64_t>(d.cols, 1) * tel, 16);
     size_t need[6] = {0, 0, 0, 0, 0, 0};
+    const int64_t Hb = d.rows * std::max(d.batch, 1);   // grid / table rows (batched FS images)
     if (seq_func(d.func)) {
       need[0] = d.rows * seq_elt_bytes(d.func);
       need[1] = d.cols * seq_elt_bytes(d.func);
     } else {
-      need[2] = d.rows * gdp;
+      need[2] = Hb * gdp;
     }
     need[3] = (d.outputs & LDDP_OUT_LAST_ROW) ? d.cols * cell_bytes(d.func) : 0;
     need[4] = (d.outputs & LDDP_OUT_LAST_COL) ? d.rows * cell_bytes(d.func) : 0;
-    need[5] = (d.outputs & LDDP_OUT_TABLE) ? d.rows * tdp + 16 : 16;
+    need[5] = (d.outputs & LDDP_OUT_TABLE) ? Hb * tdp + 16 : 16;
     for (int k = 0; k < 6; ++k) {
       if (need[k] > pl->stage_bytes[k]) {
         if (pl->stage[k]) cudaFree(pl->stage[k]);
@@ -923,7 +939,7 @@ lddp_status lddp_fill_host(lddp_plan_t pl, const lddp_inputs* hin, const lddp_ou
     if (need[0]) { CUDA_TRY(cudaMemcpyAsync(pl->stage[0], hin->a, need[0], cudaMemcpyHostToDevice, s)); din.a = pl->stage[0]; }
     if (need[1]) { CUDA_TRY(cudaMemcpyAsync(pl->stage[1], hin->b, need[1], cudaMemcpyHostToDevice, s)); din.b = pl->stage[1]; }
     if (need[2]) {
-      CUDA_TRY(cudaMemcpy2DAsync(pl->stage[2], gdp, hin->grid, hin->grid_pitch * gel, d.cols * gel, d.rows,
+      CUDA_TRY(cudaMemcpy2DAsync(pl->stage[2], gdp, hin->grid, hin->grid_pitch * gel, d.cols * gel, Hb,
                                  cudaMemcpyHostToDevice, s));
       din.grid = pl->stage[2];
       din.grid_pitch = (int64_t)(gdp / gel);
@@ -950,7 +966,7 @@ lddp_status lddp_fill_host(lddp_plan_t pl, const lddp_inputs* hin, const lddp_ou
     if (need[3]) CUDA_TRY(cudaMemcpyAsync(hout->last_row, pl->stage[3], need[3], cudaMemcpyDeviceToHost, s));
     if (need[4]) CUDA_TRY(cudaMemcpyAsync(hout->last_col, pl->stage[4], need[4], cudaMemcpyDeviceToHost, s));
     if ((d.outputs & LDDP_OUT_TABLE) && d.rows > 0 && d.cols > 0)
-      CUDA_TRY(cudaMemcpy2DAsync(hout->table, hout->table_pitch * tel, pl->stage[5], tdp, d.cols * tel, d.rows,
+      CUDA_TRY(cudaMemcpy2DAsync(hout->table, hout->table_pitch * tel, pl->stage[5], tdp, d.cols * tel, Hb,
                                  cudaMemcpyDeviceToHost, s));
     CUDA_TRY(cudaStreamSynchronize(s));
     return lddp_status_check(pl, ws, stream);
@@ -1006,6 +1022,10 @@ static void plan_share(lddp_plan_t pl, int32_t nranks, int32_t rank, int64_t* lo
     if (H == 0 || W == 0) dlo = dhi = 0;
     *lo = dlo;
     *hi = std::max(dlo, dhi);
+  } else if (pl->kind == 0 && pl->fsk) {
+    const int64_t B = std::max(d.batch, 1);   // batched FS: images
+    *lo = (int64_t)rank * B / nranks;
+    *hi = (int64_t)(rank + 1) * B / nranks;
   } else if (pl->kind == 1 && pl->cb_variant >= 0) {
     const int64_t BW = pl->cb_bw;
     const int64_t NB = (W + BW - 1) / BW;
@@ -1028,13 +1048,13 @@ lddp_status lddp_plan_partition(lddp_plan_t pl, int32_t nranks, int32_t rank, in
 lddp_status lddp_comm_create(lddp_plan_t pl, int32_t nranks, int32_t rank, lddp_comm_t* out) {
   if (pl == nullptr || out == nullptr) return fail(LDDP_ERR_INVALID_ARG, "NULL argument");
   if (nranks < 1 || rank < 0 || rank >= nranks) return fail(LDDP_ERR_INVALID_ARG, "bad rank %d / %d", rank, nranks);
-  const bool chains = pl->kind == 2;   // inverted-L / mInverted-L: diagonal shares, no exchange
+  const bool chains = pl->kind == 2 || (pl->kind == 0 && pl->fsk);   // inverted-L / batched FS: shares, no exchange
   const bool rows = pl->kind == 1;     // prev-row: column strips, two-way trapezoid halos
   if (rows && pl->cb_variant < 0)
     return fail(LDDP_ERR_UNSUPPORTED, "multi-GPU prev-row needs the column-block kernel (cols %% 4 == 0)");
   if (!chains && !rows && ((pl->kind != 3 && pl->kind != 4) || pl->desc.category != LDDP_CAT_ANTI_DIAGONAL))
     return fail(LDDP_ERR_UNSUPPORTED, "multi-GPU: anti-diagonal LCS / Levenshtein / DTW (column strips), prev-row "
-                "(column strips, two-way halos) or inverted-L / mInverted-L (diagonal shares)");
+                "(column strips, two-way halos), inverted-L / mInverted-L (diagonal shares) or FS (image shares)");
   if (!chains && pl->desc.cols < nranks) return fail(LDDP_ERR_SHAPE, "cols < nranks");
   DeviceGuard dg(pl->desc.device);
   lddp_comm_s* c = new (std::nothrow) lddp_comm_s();
@@ -1175,13 +1195,30 @@ lddp_status lddp_fill_multi(lddp_plan_t pl, const lddp_inputs* in, const lddp_ou
     if (c->plan != pl) return fail(LDDP_ERR_INVALID_ARG, "comm was created for another plan");
     lddp_status st = check_inputs(pl, in, out);
     if (st != LDDP_OK) return st;
-    if (pl->kind != 2 && c->rank < c->nranks - 1 && c->next == nullptr)
+    const bool shares = pl->kind == 2 || (pl->kind == 0 && pl->fsk);   // no exchange between ranks
+    if (!shares && c->rank < c->nranks - 1 && c->next == nullptr)
       return fail(LDDP_ERR_COMM, "rank %d is not connected to rank %d", c->rank, c->rank + 1);
-    if (pl->kind != 2 && c->rank > 0 && c->prev == nullptr)
+    if (!shares && c->rank > 0 && c->prev == nullptr)
       return fail(LDDP_ERR_COMM, "rank %d is not connected to rank %d", c->rank, c->rank - 1);
     DeviceGuard dg(pl->desc.device);
     cudaStream_t s = (cudaStream_t)stream;
     const lddp_desc& d = pl->desc;
+    if (pl->kind == 0 && pl->fsk) {
+      // Batched FS (image-parallel): rank g fills images [g B / P, (g+1) B / P) of the batch
+      // with one launch; images are independent, so nothing crosses ranks (weak scaling).
+      int64_t b0 = 0, b1 = 0;
+      plan_share(pl, c->nranks, c->rank, &b0, &b1);
+      c->fills += 1;
+      if (b1 <= b0 || d.rows == 0 || d.cols == 0) return LDDP_OK;
+      st = ensure_own_ws(pl, &ws, s);
+      if (st != LDDP_OK) return st;
+      FillParams p;
+      fill_common(pl, in, out, ws, p);
+      p.grid = static_cast<const uint8_t*>(in->grid) + b0 * d.rows * in->grid_pitch;
+      p.table = static_cast<uint8_t*>(out->table) + b0 * d.rows * out->table_pitch;
+      p.batch = (int32_t)(b1 - b0);
+      return launch(pl, p, s);
+    }
     if (pl->kind == 2) {
       // Inverted-L (and its mirror twin): every diagonal chain is independent ([L203]); rank g
       // fills a contiguous share of the diagonals holding ~1/P of the cells, writing its chains'

@@ -56,6 +56,7 @@ struct FillParams {
   int32_t spin_polls;       // polls before a waiting warp starts to back off (env LDDP_SPIN)
   int32_t debug;            // env LDDP_DEBUG bits (development): 1 = adiag warps without handoffs
   int32_t workers;          // lcs16: persistent strip workers (warps); extra warps of the last CTA idle
+  int32_t batch;            // fsk: independent images stacked along the rows (>= 1); claims are (strip, image) pairs
   int64_t diag_lo, diag_hi; // inverted-L: this rank's diagonals d = j - i in [diag_lo, diag_hi)
   // prev-row multi-GPU (column strips with two-way trapezoid halos, Table II case 2): edge pairs
   // [8 slots: fill parity x band mod 4][HB] exchanged with the neighbour ranks through the comm windows

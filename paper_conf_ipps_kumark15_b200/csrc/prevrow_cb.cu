@@ -832,19 +832,10 @@ static cudaError_t cb_dispatch(int variant, const FillParams& p, int nw, bool qu
   switch (variant) {
     case 0: return cb_launch<F, 8, 64, 48>(p, nw, query, out, s);   // BW 128
     case 1: return cb_launch<F, 8, 32, 48>(p, nw, query, out, s);
-    case 2: return cb_launch<F, 12, 48, 40>(p, nw, query, out, s);
-    case 3: return cb_launch<F, 16, 64, 32>(p, nw, query, out, s);
-    case 4: return cb_launch<F, 8, 64, 96>(p, nw, query, out, s);
     case 5: return cb_launch<F, 4, 32, 64>(p, nw, query, out, s);   // BW 64
-    case 6: return cb_launch<F, 4, 32, 64, 1>(p, nw, query, out, s);   // BW 64, bulk TMA rows
-    case 7: return cb_launch<F, 8, 64, 48, 1>(p, nw, query, out, s);   // BW 128, bulk TMA rows
     case 8: return cb_launch<F, 4, 32, 96, 2>(p, nw, query, out, s);   // BW 64, 2-D tensor TMA, 32-row groups
-    case 9: return cb_launch<F, 8, 64, 96, 2>(p, nw, query, out, s);   // BW 128, 2-D tensor TMA
     case 10: return gh_launch<F, 4, 32, 64, 4>(p, nw, query, out, s);  // BW 64, lane ghosts: SHFL every 4 rows
-    case 11: return gh_launch<F, 8, 64, 48, 8>(p, nw, query, out, s);  // BW 128, lane ghosts every 8 rows
-    case 12: return gh_launch<F, 8, 64, 48, 4>(p, nw, query, out, s);  // BW 128, lane ghosts every 4 rows
     case 13: return cb_launch<F, 2, 16, 64>(p, nw, query, out, s);      // BW 32, 8-byte segments, 1024 warps for C4
-    case 14: return cb_launch<F, 2, 16, 96>(p, nw, query, out, s);      // BW 32, deeper ring
     case 17: return cb_launch<F, 6, 48, 48>(p, nw, query, out, s);      // BW 96, exchange every 48 rows
     case 18: return cb_launch<F, 6, 48, 32>(p, nw, query, out, s);      // BW 96, 32-row ring
     default: return cudaErrorInvalidValue;

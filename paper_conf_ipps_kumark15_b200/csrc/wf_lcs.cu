@@ -3,16 +3,8 @@
 namespace lddp {
 int wf_dispatch_lcs(int op, int variant, bool table, const FillParams* p, int grid, cudaStream_t s) {
   LDDP_WF_CASE(CellLCS, WF_A_R4_S0, 4, 0, 2, false)
-  LDDP_WF_CASE(CellLCS, WF_A_R4_S1, 4, 1, 1, false)
   LDDP_WF_CASE(CellLCS, WF_A_R2_S1, 2, 1, 1, false)
   LDDP_WF_CASE(CellLCS, WF_A_R8_S1, 8, 1, 1, false)
-  LDDP_WF_CASE(CellLCS, WF_A_R8_S0, 8, 0, 2, false)
-  LDDP_WF_CASE(CellLCS, WF_A_R4_E1, 4, 0, 1, false)
-  LDDP_WF_CASE(CellLCS, WF_A_R16_S0, 16, 0, 2, false)
-  LDDP_WF_CASE(CellLCS, WF_A_R8_E3, 8, 0, 3, false)
-  LDDP_WF_CASE_G(CellLCS, WF_A_R8_G4, 8, 1, 1, false, 4)
-  LDDP_WF_CASE_G(CellLCS, WF_A_R8_G2, 8, 1, 1, false, 2)
-  LDDP_WF_CASE_G(CellLCS, WF_A_R16_G4, 16, 1, 1, false, 4)
   LDDP_WF_CASE(CellLCS, WF_A_R4_S0, 4, 0, 2, true)
   LDDP_WF_CASE(CellLCS, WF_K_R1, 1, 2, 2, false)
   LDDP_WF_CASE(CellLCS, WF_K_R2, 2, 2, 2, false)

@@ -3,7 +3,6 @@
 namespace lddp {
 int wf_dispatch_min2plus(int op, int variant, bool table, const FillParams* p, int grid, cudaStream_t s) {
   LDDP_WF_CASE(CellMin2Plus, WF_A_R4_S0, 4, 0, 2, false)
-  LDDP_WF_CASE(CellMin2Plus, WF_A_R4_S1, 4, 1, 1, false)
   LDDP_WF_CASE(CellMin2Plus, WF_A_R2_S1, 2, 1, 1, false)
   LDDP_WF_CASE(CellMin2Plus, WF_A_R8_S1, 8, 1, 1, false)
   LDDP_WF_CASE(CellMin2Plus, WF_A_R4_S0, 4, 0, 2, true)

@@ -50,7 +50,7 @@ class lddp_desc(ctypes.Structure):
                 ("func", ctypes.c_int32), ("outputs", ctypes.c_uint32), ("param_c", ctypes.c_int32),
                 ("device", ctypes.c_int32), ("tile_rows", ctypes.c_int32),
                 ("tile_warps", ctypes.c_int32), ("band_rows", ctypes.c_int32),
-                ("grid_ctas", ctypes.c_int32), ("reserved", ctypes.c_int32 * 3)]
+                ("grid_ctas", ctypes.c_int32), ("batch", ctypes.c_int32), ("reserved", ctypes.c_int32 * 2)]
 
 
 class lddp_inputs(ctypes.Structure):
@@ -235,7 +235,7 @@ class Plan:
     """A plan plus its workspace (torch uint8 tensor on the plan's device)."""
 
     def __init__(self, func, category, rows, cols, outputs, param_c=1, device=0, tile_rows=0,
-                 grid_ctas=0, band_rows=0):
+                 grid_ctas=0, band_rows=0, batch=0):
         import torch
         self.func = FUNCS[func] if isinstance(func, str) else int(func)
         self.category = CATEGORIES[category] if isinstance(category, str) else int(category)
@@ -244,7 +244,7 @@ class Plan:
         self.desc = lddp_desc(rows=self.rows, cols=self.cols, category=self.category, func=self.func,
                               outputs=self.outputs, param_c=int(param_c), device=self.device,
                               tile_rows=int(tile_rows), tile_warps=0, band_rows=int(band_rows),
-                              grid_ctas=int(grid_ctas))
+                              grid_ctas=int(grid_ctas), batch=int(batch))
         self.handle = lddp_plan(self.desc)
         self.ws_bytes = lddp_plan_workspace_size(self.handle)
         self.ws = torch.zeros(max(self.ws_bytes, 64), dtype=torch.uint8, device=f"cuda:{self.device}")

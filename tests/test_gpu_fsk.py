@@ -35,8 +35,7 @@ def fsk_env():
             os.environ[k] = v
 
 
-@pytest.mark.parametrize("w,e,r", [(4, 0, 1), (4, 1, 1), (4, 2, 1), (2, 0, 1), (2, 1, 1), (2, 2, 1),
-                                   (2, 0, 2), (2, 1, 2), (1, 0, 2), (1, 1, 2), (1, 1, 1), (1, 0, 1), (1, 0, 3)])
+@pytest.mark.parametrize("w,e,r", [(1, 1, 1), (1, 0, 1), (1, 2, 1), (1, 1, 2), (1, 0, 2), (4, 1, 1), (2, 1, 1)])
 @pytest.mark.parametrize("shape", FS_SHAPES)
 @pytest.mark.parametrize("kind", ["ramp", "uniform"])
 def test_fsk_parity(fsk_env, w, e, r, shape, kind):

@@ -36,7 +36,7 @@ def cb_env():
             os.environ[k] = v
 
 
-@pytest.mark.parametrize("variant,warps", [(0, 2), (1, 1), (2, 2), (3, 1), (4, 2), (0, 4), (5, 4), (5, 2), (6, 2), (6, 4), (7, 2), (7, 1), (8, 2), (8, 1), (8, 4), (9, 2), (10, 2), (10, 1), (10, 4), (11, 2), (12, 2), (13, 2), (13, 4), (13, 8), (14, 4), (17, 4), (17, 2), (18, 4)])
+@pytest.mark.parametrize("variant,warps", [(0, 2), (1, 1), (0, 4), (5, 4), (5, 2), (8, 2), (8, 1), (8, 4), (10, 2), (10, 1), (10, 4), (13, 2), (13, 4), (13, 8), (17, 4), (17, 2), (18, 4)])
 @pytest.mark.parametrize("shape", CB_SHAPES)
 def test_minpath3_cb(cb_env, variant, warps, shape):
     cb_env(variant, warps)
@@ -54,7 +54,7 @@ def test_minpath3_cb(cb_env, variant, warps, shape):
         np.testing.assert_array_equal(got["table"], ref.table)
 
 
-@pytest.mark.parametrize("variant", [0, 1, 3, 5, 6, 7, 8, 9, 10, 11, 12, 13])
+@pytest.mark.parametrize("variant", [0, 1, 5, 8, 10, 13])
 @pytest.mark.parametrize("shape", [(1000, 1000), (300, 2052)])
 def test_min2plus_diagmaxplus_cb(cb_env, variant, shape):
     cb_env(variant, 2)

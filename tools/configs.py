@@ -1,6 +1,6 @@
 """The BASELINE.json workloads C1-C5 and the two synthetic-f
 workloads of SURVEY §8(d) "(iL)" / [L298] (C6 inverted-L diagonal max-plus, C7 horizontal
-min2-plus): shapes, f, category and the seeded input recipe.  Shared by bench.py,
+min2-plus) and C8 (batched FS, §8(f)#3): shapes, f, category and the seeded input recipe.  Shared by bench.py,
 tools/make_bench_refs.py and the full-size tests."""
 import os
 import sys
@@ -31,6 +31,13 @@ def _fs(n):
     return make
 
 
+def _fs_batch(n, B):
+    def make(seed):
+        import numpy as np
+        return {"grid": np.concatenate([inputs.gen_image(seed + b, n, n, "ramp") for b in range(B)], axis=0)}
+    return make
+
+
 def _minpath(n):
     def make(seed):
         return {"grid": inputs.gen_costs(seed, n, n)}
@@ -57,6 +64,10 @@ CONFIGS = {
     "C6": {"func": "diagmaxplus", "category": "inverted_l", "rows": 32768, "cols": 32768, "make": _init(32768),
            "param_c": 1,
            "desc": "inverted-L synthetic f = max(init, UL) + 1 [L298] on a 32768x32768 int32 grid (SURVEY 8(d) iL)"},
+    "C8": {"func": "fs", "category": "knight_move", "rows": 8 * 8192, "cols": 8192, "batch": 8, "img_rows": 8192,
+           "make": _fs_batch(8192, 8),
+           "desc": "batched FS: 8 independent 8192x8192 images (seeds 0..7, C3's recipe) in one launch, "
+                   "image-parallel (SURVEY 8(f)#3, R21); rows = the stacked batch"},
     "C7": {"func": "min2plus", "category": "prev_row", "rows": 32768, "cols": 32768, "make": _init(32768),
            "param_c": 1,
            "desc": "horizontal case-1 synthetic f = min(UL, U) + 1 [L298] (H1) on a 32768x32768 int32 grid"},

@@ -42,7 +42,9 @@ def main():
             score = float(r.score) if cfg["func"] == "dtw" else int(r.score)
             ent = {"score": score, "last_row_sha256": digest(r.last_row), "last_col_sha256": digest(r.last_col)}
         elif cfg["func"] == "fs":
-            img = oracle.fs(x["grid"])
+            ir = cfg.get("img_rows", cfg["rows"])   # batched FS: each image of the stack on its own
+            g = x["grid"]
+            img = np.concatenate([oracle.fs(g[k:k + ir]) for k in range(0, g.shape[0], ir)], axis=0)
             ent = {"image_sha256": digest(img), "white_fraction": float((img == 255).mean())}
         elif cfg["func"] == "minpath3":
             r = oracle.minpath3(x["grid"])
