@@ -471,7 +471,8 @@ lddp_status launch(lddp_plan_t pl, const FillParams& p, cudaStream_t s) {
     }
     return LDDP_OK;
   } else {
-    e = lddp::launch_invl(pl->desc.func, p, pl->grid, pl->mirror, s);
+    e = env_int("LDDP_INVL_TMA", 1) ? lddp::launch_invl_tma(p, pl->mirror, pl->sms, s) : cudaErrorNotSupported;
+    if (e == cudaErrorNotSupported) e = lddp::launch_invl(pl->desc.func, p, pl->grid, pl->mirror, s);
   }
   if (e != cudaSuccess) return cuda_fail(e, "kernel launch");
   return LDDP_OK;
@@ -1237,7 +1238,8 @@ lddp_status lddp_fill_multi(lddp_plan_t pl, const lddp_inputs* in, const lddp_ou
       const int64_t warps = (p.diag_hi - p.diag_lo + 31) / 32;
       const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((warps + kInvlThreads / 32 - 1) / (kInvlThreads / 32),
                                                                    (int64_t)pl->sms * 16));
-      cudaError_t e = lddp::launch_invl(d.func, p, grid, pl->mirror, s);
+      cudaError_t e = env_int("LDDP_INVL_TMA", 1) ? lddp::launch_invl_tma(p, pl->mirror, pl->sms, s) : cudaErrorNotSupported;
+      if (e == cudaErrorNotSupported) e = lddp::launch_invl(d.func, p, grid, pl->mirror, s);
       if (e != cudaSuccess) return cuda_fail(e, "kernel launch");
       return LDDP_OK;
     }

@@ -82,6 +82,8 @@ cudaError_t launch_traceback(int func, const void* a, const void* b, const void*
 // Inverted-L kernel (invl.cu); mirror: read / write the grid with column j <-> W-1-j (the
 // mInverted-L twin [L111]).
 cudaError_t launch_invl(int func, const FillParams& p, int grid, bool mirror, cudaStream_t stream);
+// TMA-staged inverted-L (no TABLE, 16-byte aligned grid, pitch % 4 == 0): cudaErrorNotSupported otherwise
+cudaError_t launch_invl_tma(const FillParams& p, bool mirror, int sms, cudaStream_t stream);
 // dst (cols x rows) = transpose of src (rows x cols), 32-bit elements, pitches in elements.
 cudaError_t launch_transpose_i32(const int32_t* src, int64_t spitch, int32_t* dst, int64_t dpitch, int64_t rows,
                                  int64_t cols, cudaStream_t s);
