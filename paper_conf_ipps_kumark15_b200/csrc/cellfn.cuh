@@ -192,9 +192,9 @@ struct CellFS {
     v = __fadd_rn(v, __fmul_rn(U, 0.3125f));
     v = __fadd_rn(v, __fmul_rn(UR, 0.1875f));
     v = __fadd_rn(v, __fmul_rn(L, 0.4375f));
-    // threshold as a register mask (FSET), not a predicate (FSETP -> predicated use costs ~13
-    // cycles on the error chain): m = v >= 128 ? ~0 : 0; e = v - (m & 255.0f), exactly the
-    // oracle's v - 255 or v (v - (+0) == v for every v, -0 included)
+    // threshold as a register mask (set.ge.u32.f32) rather than a branch-like select of two
+    // results: m = v >= 128 ? ~0 : 0; e = v - (m & bits(255.0f)), exactly the oracle's v - 255 or
+    // v - (+0) = v.  (An integer-compare formulation on the bits measured slower: C3 1.57 -> 1.62 ms.)
     uint32_t m;
     asm("set.ge.u32.f32 %0, %1, 128.0;" : "=r"(m) : "f"(v));
     o = (uint8_t)(m & 255u);

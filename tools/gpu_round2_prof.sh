@@ -28,6 +28,11 @@ SKIP=0 cap x_transpose transpose python tools/prof_extra.py
 SKIP=0 cap x_invl_mirror invl python tools/prof_extra.py
 for f in $O/prof_*.ncu-rep; do
   b=$(basename $f .ncu-rep)
-  ncu -i $f --page raw --csv > $O/${b}_raw.csv 2>/dev/null
-  ncu -i $f --page source --csv --print-source sass > $O/${b}_sass.csv 2>/dev/null
+  python tools/ncu_summary.py $f > $O/${b}.json 2>/dev/null
+  ncu -i $f --page raw --csv 2>/dev/null | gzip > $O/${b}_raw.csv.gz
 done
+# keep the two headline reports (C5 lcs16, C4 prevrow_cb); the rest are summarised above
+for f in $O/prof_*.ncu-rep; do
+  case $f in *c5_lcs16*|*c4_prevrow_cb*) ;; *) rm -f $f ;; esac
+done
+du -sh $O
