@@ -442,9 +442,9 @@ def scaling_model(ms1, plan, cols):
     time, at the same per-chunk cost on any GPU count).  The per-chunk time t and the strip lag L
     (2E + 1 chunks of structure + ~0.9 chunk of handoff latency, tools/l16_trace.py) are
     calibrated on the measured N = 1 time; t_link = one NVLink store + flag hop (~2 us, assumed)."""
-    S, NQ, E = plan["strips"], plan["chunks"], plan["extra_lag"]
     if plan.get("kernel") != "lcs16":
         return None
+    S, NQ, E = plan["strips"], plan["chunks"], plan["extra_lag"]
     L = 2 * E + 1.9
     t = ms1 / (NQ + 2 * E + (S - 1) * L)
     t_link = 2e-3

@@ -216,6 +216,9 @@ struct lddp_plan_s {
   int cb_bw;         // its own columns per warp (block width)
   int cb_nw;         // warps per CTA
   int cb_nblocks;    // column blocks (one warp each)
+  int hx_variant;    // hierarchical-exchange kernel (prevrow_hx.cu, no TABLE): -1 = not usable
+  int hx_cw;         // its own columns per CTA
+  int hx_ctas;       // CTAs (one per SM at most)
   // Floyd-Steinberg lane-systolic kernel (fsk.cu): used when the widths / pitches allow
   bool fsk;
   // symmetric twins: mInverted-L = the inverted-L kernel on the mirrored grid; Vertical = a
@@ -420,6 +423,10 @@ lddp_status launch(lddp_plan_t pl, const FillParams& p, cudaStream_t s) {
     q.strip_rows = 192;
     q.bnd_stride = (int64_t)std::max((q.cols + 31) / 32, 1) * 32;
     e = lddp::ad_lcs_r6e2w1(q, std::min(q.nstrips, pl->sms * 8), s);
+  } else if (pl->kind == 1 && pl->hx_variant >= 0 && p.table == nullptr && p.grid_pitch % 4 == 0 &&
+             p.grid_pitch < ((int64_t)1 << 29) && ((reinterpret_cast<uintptr_t>(p.grid) & 15) == 0)) {
+    int dummy[3];
+    e = lddp::launch_prevrow_hx(pl->desc.func, pl->hx_variant, p, false, dummy, s);
   } else if (pl->kind == 1 && pl->cb_variant >= 0 && (p.grid_pitch % 4 == 0) &&
              ((reinterpret_cast<uintptr_t>(p.grid) & 15) == 0)) {
     FillParams q = p;
@@ -772,6 +779,33 @@ lddp_status lddp_plan(const lddp_desc* desc, lddp_plan_t* out) {
           cudaGetLastError();
         }
       }
+      // Hierarchical-exchange kernel for SCORE / LAST_ROW fills: CTAs of four
+      // warps exchange inner halos through shared memory, outer halos through L2 every HBO rows.
+      // desc.band_rows keeps selecting the prev-row_cb band height (it is that kernel's knob).
+      pl->hx_variant = -1;
+      // measured defaults (tools/gpu_hx5.sh, one B200): MIN_PATH3 lane ghosts + 96-row ring (C4
+      // 2.01 -> 1.64 ms); single-neighbour-pair f's without ghosts (C7 2.33 -> 1.67 ms)
+      const int hxv = env_int("LDDP_HX_VARIANT", d.func == LDDP_F_MIN_PATH3 ? 4 : 2);
+      if (hxv >= 0 && d.band_rows <= 0 && !(d.outputs & LDDP_OUT_TABLE) && d.cols > 0 && d.rows > 0 &&
+          d.cols % 4 == 0 && d.rows < (int64_t)1 << 30) {
+        int q[3] = {0, 0, 0};
+        FillParams dummy{};
+        if (lddp::launch_prevrow_hx(d.func, hxv, dummy, true, q, nullptr) == cudaSuccess && q[0] > 0) {
+          const int64_t ctas = (d.cols + q[0] - 1) / q[0];
+          if (q[1] > 0 && ctas <= (int64_t)q[1] * pl->sms) {
+            pl->hx_variant = hxv;
+            pl->hx_cw = q[0];
+            pl->hx_ctas = (int)ctas;
+            // workspace: per-CTA row minima + outer edge pairs [CTA][4 slots][2 sides][HBO] x 8 B
+            const size_t prog = align_up(64 + (size_t)ctas * 4, 256);
+            pl->off_prog = 64;
+            pl->off_bnd = std::max(pl->off_bnd, prog);
+            pl->ws_bytes = std::max(pl->ws_bytes, pl->off_bnd + (size_t)ctas * 4 * 2 * q[2] * 8);
+          }
+        } else {
+          cudaGetLastError();
+        }
+      }
     } else if (d.category == LDDP_CAT_VERTICAL) {
       // Vertical = transpose of Horizontal [L111]: transpose the grid into the workspace, run the
       // prev-row plan of the transposed problem (its last row = our last column, its score =
@@ -841,6 +875,14 @@ lddp_status lddp_plan_describe(lddp_plan_t pl, char* buf, size_t len) {
     return LDDP_OK;
   }
   const bool cb = pl->kind == 1 && pl->cb_variant >= 0;
+  if (pl->kind == 1 && pl->hx_variant >= 0) {
+    snprintf(buf, len,
+             "{\"kernel\": \"prevrow_hx\", \"variant\": %d, \"warps\": 4, \"grid\": %d, \"sms\": %d, "
+             "\"occupancy\": 1, \"cta_cols\": %d, \"workspace_bytes\": %zu, "
+             "\"fallback\": \"prevrow_cb variant %d (TABLE, multi-GPU, unaligned grids)\"}",
+             pl->hx_variant, pl->hx_ctas, pl->sms, pl->hx_cw, pl->ws_bytes, pl->cb_variant);
+    return LDDP_OK;
+  }
   if (pl->kind == 0 && pl->fsk) {
     snprintf(buf, len,
              "{\"kernel\": \"fsk\", \"variant\": -1, \"rows_per_lane\": %d, \"skew\": 2, \"extra_lag\": %d, "

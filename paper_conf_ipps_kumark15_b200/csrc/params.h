@@ -74,6 +74,10 @@ cudaError_t launch_prevrow(int func, const FillParams& p, int grid, cudaStream_t
 // per warp, out[1] = co-resident CTAs per SM (nothing launched).
 cudaError_t launch_prevrow_cb(int func, int variant, const FillParams& p, int nw, bool query, int* out,
                               cudaStream_t stream);
+// Hierarchical-exchange prev-row kernel (prevrow_hx.cu; SCORE / LAST_ROW, one GPU, cooperative
+// launch).  query: out[0] = own columns per CTA, out[1] = co-resident CTAs per SM, out[2] = outer
+// halo HBO (edge pairs per CTA side).
+cudaError_t launch_prevrow_hx(int func, int variant, const FillParams& p, bool query, int* out, cudaStream_t stream);
 // Floyd-Steinberg lane-systolic knight kernel (fsk.cu): W warps per CTA, E extra lane lag.
 cudaError_t launch_fsk(const FillParams& p, int W, int E, int R, int grid, cudaStream_t stream);
 // Traceback of a LCS / Levenshtein / DTW table (traceback.cu): one thread, O(m + n).

@@ -21,12 +21,13 @@ CB_SHAPES = [(1, 4), (2, 8), (63, 132), (64, 256), (65, 260), (129, 388), (1000,
 
 @pytest.fixture
 def cb_env():
-    keys = ("LDDP_CB_VARIANT", "LDDP_CB_WARPS")
+    keys = ("LDDP_CB_VARIANT", "LDDP_CB_WARPS", "LDDP_HX_VARIANT")
     old = {k: os.environ.get(k) for k in keys}
 
     def set_(variant, warps):
         os.environ["LDDP_CB_VARIANT"] = str(variant)
         os.environ["LDDP_CB_WARPS"] = str(warps)
+        os.environ["LDDP_HX_VARIANT"] = "-1"   # SCORE / LAST_ROW fills would take prevrow_hx
 
     yield set_
     for k, v in old.items():

@@ -25,11 +25,18 @@ def main():
     ap.add_argument("--variant", type=int, nargs="*", default=[-1])
     ap.add_argument("--grid", type=int, nargs="*", default=[0])
     ap.add_argument("--reps", type=int, default=5)
+    ap.add_argument("--env", nargs="*", default=[], help="KEY=v1,v2,... swept (outer product)")
     args = ap.parse_args()
     from paper_conf_ipps_kumark15_b200 import lddp
     dev = torch.device("cuda", 0)
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
-    for name in args.configs:
+    import itertools
+    keys = [e.split("=")[0] for e in args.env]
+    vals = [e.split("=")[1].split(",") for e in args.env]
+    for combo in (itertools.product(*vals) if keys else [()]):
+      for k, v in zip(keys, combo):
+        os.environ[k] = v
+      for name in args.configs:
         for rows in args.rows:
             for var in args.variant:
                 for g in args.grid:
@@ -44,12 +51,12 @@ def main():
                         ms, per, _, _ = bench.time_device(pb, lddp, args.reps, 2, dev, 1, flush)
                         par = bench.check_result(name, pb)
                         cells = CONFIGS[name]["rows"] * CONFIGS[name]["cols"]
-                        print(json.dumps({"cfg": name, "rows": rows, "variant": var, "grid": g,
+                        print(json.dumps({"env": dict(zip(keys, combo)), "cfg": name, "rows": rows, "variant": var, "grid": g,
                                           "ms": round(ms, 4), "min": round(min(per), 4),
                                           "gcups": round(cells / ms / 1e6, 1), "parity": par.get("match"),
                                           "plan": json.loads(pb["plan"].info)}), flush=True)
                     except Exception as e:  # keep going
-                        print(json.dumps({"cfg": name, "rows": rows, "variant": var, "error": str(e)[:300]}), flush=True)
+                        print(json.dumps({"env": dict(zip(keys, combo)), "cfg": name, "rows": rows, "variant": var, "error": str(e)[:300]}), flush=True)
                     torch.cuda.empty_cache()
                     print(f"# {name} took {time.time() - t0:.1f}s", flush=True)
 
