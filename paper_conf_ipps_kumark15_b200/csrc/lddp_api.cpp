@@ -783,9 +783,9 @@ lddp_status lddp_plan(const lddp_desc* desc, lddp_plan_t* out) {
       // warps exchange inner halos through shared memory, outer halos through L2 every HBO rows.
       // desc.band_rows keeps selecting the prev-row_cb band height (it is that kernel's knob).
       pl->hx_variant = -1;
-      // measured defaults (tools/gpu_hx5.sh, one B200): MIN_PATH3 lane ghosts + 96-row ring (C4
-      // 2.01 -> 1.64 ms); single-neighbour-pair f's without ghosts (C7 2.33 -> 1.67 ms)
-      const int hxv = env_int("LDDP_HX_VARIANT", d.func == LDDP_F_MIN_PATH3 ? 4 : 2);
+      // measured default (tools/gpu_hx5.sh, one B200): variant 2 (no lane ghosts, 64-row ring):
+      // C4 2.00 -> 1.53 ms, C7 2.33 -> 1.55 ms
+      const int hxv = env_int("LDDP_HX_VARIANT", 2);
       if (hxv >= 0 && d.band_rows <= 0 && !(d.outputs & LDDP_OUT_TABLE) && d.cols > 0 && d.rows > 0 &&
           d.cols % 4 == 0 && d.rows < (int64_t)1 << 30) {
         int q[3] = {0, 0, 0};

@@ -273,6 +273,16 @@ __global__ void __launch_bounds__(NW * 32, 1) prevrow_hx_kernel(const FillParams
   const bool pub_r = own && e0 >= A + CW - HBO && e0 < A + CW;     // CTA c+1 reads these
   const bool get_l = w == 0 && lhalo && c > 0;
   const bool get_r = w == NW - 1 && rhalo && c + 1 < nc;
+  const bool pub = pub_l || pub_r, get = get_l || get_r;
+  const bool ihalo = !own && !((w == 0 && lhalo) || (w == NW - 1 && rhalo));   // inner halo lane
+  // this lane's pair addresses in slot 0 (slot s adds s * 2 * HBO): own edge columns it publishes,
+  // neighbour columns it polls
+  uint64_t* const pubp = edges + ((size_t)c * 8 + (pub_l ? 0 : 1)) * HBO + (pub_l ? e0 - A : e0 - (A + CW - HBO));
+  const uint64_t* const getp = get_l ? edges + ((size_t)(c - 1) * 8 + 1) * HBO + (e0 - (A - HBO))
+                                     : edges + ((size_t)(c + 1) * 8 + 0) * HBO + (e0 - (A + CW));
+  const uint32_t xsa = xs0 + (uint32_t)(xidx * 4);
+  uint32_t xpar = 0;
+  int kin = 0, ob = 0;   // inner band within the outer band, outer band
   bool aborted = false;
 
   // development trace (LDDP_TRACE, tools/hx_trace.py): CTA trace_chunks, lane 0 of every warp,
@@ -298,32 +308,31 @@ __global__ void __launch_bounds__(NW * 32, 1) prevrow_hx_kernel(const FillParams
     if (r0 + HBI >= H) break;
 
     // ---- inner band boundary: own columns -> shared exchange row, halos <- neighbours
-    const int band = r0 / HBI;
-    const uint32_t xs = xs0 + (uint32_t)((band & 1) * NW * EXT * 4);
-    if (own) hx::sts128(xs + (uint32_t)(xidx * 4), make_int4(st.x[GH], st.x[GH + 1], st.x[GH + 2], st.x[GH + 3]));
-    const bool outer = ((r0 + HBI) % HBO) == 0;
-    const int ob = (r0 + HBI) / HBO - 1;   // outer band just finished
+    const uint32_t xs = xsa + xpar;
+    xpar ^= (uint32_t)(NW * EXT * 4);
+    if (own) hx::sts128(xs, make_int4(st.x[GH], st.x[GH + 1], st.x[GH + 2], st.x[GH + 3]));
+    const bool outer = kin == HBO / HBI - 1;   // an outer band (HBO rows) ends here
+    kin = outer ? 0 : kin + 1;
     const uint32_t tag = tag0 | (((uint32_t)ob + 1u) & 0xFFFFFu);
-    if (outer && (pub_l || pub_r)) {
-      uint64_t* d = edges + (((size_t)c * 4 + (ob & 3)) * 2 + (pub_l ? 0 : 1)) * HBO +
-                    (pub_l ? e0 - A : e0 - (A + CW - HBO));
-      hx::st_pair2(d, ((uint64_t)tag << 32) | (uint32_t)st.x[GH], ((uint64_t)tag << 32) | (uint32_t)st.x[GH + 1]);
-      hx::st_pair2(d + 2, ((uint64_t)tag << 32) | (uint32_t)st.x[GH + 2], ((uint64_t)tag << 32) | (uint32_t)st.x[GH + 3]);
+    if (outer && pub) {
+      uint64_t* d = pubp + (size_t)(ob & 3) * 2 * HBO;
+      const uint64_t th = (uint64_t)tag << 32;
+      hx::st_pair2(d, th | (uint32_t)st.x[GH], th | (uint32_t)st.x[GH + 1]);
+      hx::st_pair2(d + 2, th | (uint32_t)st.x[GH + 2], th | (uint32_t)st.x[GH + 3]);
     }
-    if (!dbg_no_inner) hx::bar_named<NW * 32>();
-    const bool from_l2 = outer && (get_l || get_r) && !dbg_no_outer;
-    if (!own && !from_l2 && !((w == 0 && lhalo) || (w == NW - 1 && rhalo)) && !dbg_no_inner) {
-      const int4 v = hx::lds128(xs + (uint32_t)(xidx * 4));
-      st.x[GH] = v.x; st.x[GH + 1] = v.y; st.x[GH + 2] = v.z; st.x[GH + 3] = v.w;
+    if (!dbg_no_inner) {
+      hx::bar_named<NW * 32>();
+      if (ihalo) {
+        const int4 v = hx::lds128(xs);
+        st.x[GH] = v.x; st.x[GH + 1] = v.y; st.x[GH + 2] = v.z; st.x[GH + 3] = v.w;
+      }
     }
-    if (outer && (w == 0 || w == NW - 1)) {
-      const uint64_t* s = nullptr;
-      if (from_l2)
-        s = get_l ? edges + (((size_t)(c - 1) * 4 + (ob & 3)) * 2 + 1) * HBO + (e0 - (A - HBO))
-                  : edges + (((size_t)(c + 1) * 4 + (ob & 3)) * 2 + 0) * HBO + (e0 - (A + CW));
+    if (outer && (w == 0 || w == NW - 1) && !dbg_no_outer) {
+      const uint64_t* s = getp + (size_t)(ob & 3) * 2 * HBO;
+      const bool need = get && !aborted;
       uint64_t pr[VP];
       bool ok = true;
-      if (from_l2 && !aborted) {
+      if (need) {
         hx::ld_pair2(s, pr[0], pr[1]);
         hx::ld_pair2(s + 2, pr[2], pr[3]);
 #pragma unroll
@@ -346,16 +355,16 @@ __global__ void __launch_bounds__(NW * 32, 1) prevrow_hx_kernel(const FillParams
           if (++spins > 64 && !bo.tick(ctl, p.timeout_ns)) {
             aborted = true;
             ok = true;
-            break;
           }
         }
         aborted = __any_sync(0xffffffffu, aborted);
       }
-      if (from_l2 && !aborted) {
+      if (need && !aborted) {
 #pragma unroll
         for (int v = 0; v < VP; ++v) st.x[GH + v] = (T)(uint32_t)pr[v];
       }
     }
+    if (outer) ++ob;
     if (trc && r0 / HBI < 4096) p.trace[((r0 / HBI) * NW + w) * 2 + 1] = (uint64_t)(clock64() - tb0);
   }
   hx::wait_group<0>();
