@@ -436,6 +436,9 @@ static cudaError_t hx_dispatch(int variant, const FillParams& p, bool query, int
     case 4: return hx_launch<F, 4, 16, 96, 96, 2>(p, query, out, s);   // deeper ring
     case 5: return hx_launch<F, 4, 16, 96, 32, 2>(p, query, out, s);   // shallower ring
     case 6: return hx_launch<F, 4, 16, 64, 64, 1>(p, query, out, s);   // CW 288, no lane ghosts
+    case 7: return hx_launch<F, 4, 16, 80, 64, 1>(p, query, out, s);   // CW 256
+    case 8: return hx_launch<F, 4, 16, 96, 32, 1>(p, query, out, s);   // 32-row ring
+    case 9: return hx_launch<F, 4, 16, 96, 96, 1>(p, query, out, s);   // 96-row ring
     default: return cudaErrorInvalidValue;
   }
 }
