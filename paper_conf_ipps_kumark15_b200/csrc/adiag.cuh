@@ -60,6 +60,14 @@ __device__ __forceinline__ uint64_t ad_ld_gpu(const uint64_t* p) {
   asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
   return v;
 }
+// the same load for prefetches whose staleness the tag check catches: no memory clobber, so the
+// scheduler may still move other memory operations around it (volatile: never speculated out of
+// its predicate -- a non-volatile asm was hoisted past the bounds check)
+__device__ __forceinline__ uint64_t ad_ld_gpu_pf(const uint64_t* p) {
+  uint64_t v;
+  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p));
+  return v;
+}
 __device__ __forceinline__ void ad_st_gpu2(uint64_t* p, uint64_t a, uint64_t b) {
   asm volatile("st.relaxed.gpu.global.v2.u64 [%0], {%1, %2};" ::"l"(p), "l"(a), "l"(b) : "memory");
 }
@@ -291,10 +299,11 @@ struct AdWarp {
     }
 #pragma unroll(kAdGroupUnroll<F>)
     for (int g = 0; g < 4; ++g) {
-      // a plain L2 load (predicated, no branch in the group body); a stale pair is caught by
-      // the tag check and re-polled with a strong load in acquire_top
+      // a relaxed gpu-scope L2 load (in the memory model: it races the producer's relaxed pair
+      // store; predicated, no branch in the group body); a stale pair is caught by the tag check
+      // and re-polled in acquire_top
       if constexpr (kAdHalfPf) {
-        if (g == kAdPfGroup<F> && k + 1 < tqn) tq1 = __ldcg(reinterpret_cast<const unsigned long long*>(tqsrc) + 32 * (k + 1));
+        if (g == kAdPfGroup<F> && k + 1 < tqn) tq1 = ad_ld_gpu_pf(reinterpret_cast<const uint64_t*>(tqsrc) + 32 * (k + 1));
       }
       CC cnext[8];
       const int tau0 = 32 * k - E + 8 * g;

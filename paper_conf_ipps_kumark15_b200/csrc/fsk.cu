@@ -223,7 +223,7 @@ __global__ void __launch_bounds__(W * 32, 1) fsk_kernel(const FillParams p) {
         // the next chunk's strip-boundary pair, half a chunk ahead: late enough that the producer
         // has usually published it (a stale pair is caught by the tag check and re-polled)
         if (g == LDDP_FSK_PG && topsrc == 2 && k + 1 < NQ)
-          tq1 = __ldcg(reinterpret_cast<const unsigned long long*>(gprev) + 32 * (k + 1) + lane);
+          tq1 = ad_ld_gpu_pf(reinterpret_cast<const uint64_t*>(gprev) + 32 * (k + 1) + lane);   // relaxed.gpu: races the pair store
         float bv[8];
         float inn[R][8], injn[8];
         if (g < 3) {
