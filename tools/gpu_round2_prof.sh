@@ -17,15 +17,16 @@ cap c5_lcs16 lcs16 python bench.py --workload C5 --no-others --no-cpu --steps 1 
 cap c1_lcs16 lcs16 python bench.py --workload C1 --no-others --no-cpu --steps 1 --warmup 3
 cap c2_adiag adiag python bench.py --workload C2 --no-others --no-cpu --steps 1 --warmup 3
 cap c3_fsk fsk python bench.py --workload C3 --no-others --no-cpu --steps 1 --warmup 3
-cap c4_prevrow_cb prevrow_cb python bench.py --workload C4 --no-others --no-cpu --steps 1 --warmup 3
+cap c4_prevrow_hx prevrow_hx python bench.py --workload C4 --no-others --no-cpu --steps 1 --warmup 3
 cap c6_invl invl python bench.py --workload C6 --no-others --no-cpu --steps 1 --warmup 3
-cap c7_prevrow_cb prevrow_cb python bench.py --workload C7 --no-others --no-cpu --steps 1 --warmup 3
+cap c7_prevrow_hx prevrow_hx python bench.py --workload C7 --no-others --no-cpu --steps 1 --warmup 3
 cap c8_fsk_batch fsk python bench.py --workload C8 --no-others --no-cpu --steps 1 --warmup 3
 SKIP=0 cap x_wavefront_table wavefront python tools/prof_extra.py
 SKIP=0 cap x_traceback traceback python tools/prof_extra.py
 SKIP=0 cap x_prevrow_fallback "prevrow_kernel" python tools/prof_extra.py
 SKIP=0 cap x_transpose transpose python tools/prof_extra.py
 SKIP=0 cap x_invl_mirror invl python tools/prof_extra.py
+SKIP=0 cap x_prevrow_cb_table prevrow_cb python tools/prof_extra.py
 for f in $O/prof_*.ncu-rep; do
   b=$(basename $f .ncu-rep)
   python tools/ncu_summary.py $f > $O/${b}.json 2>/dev/null
@@ -33,6 +34,6 @@ for f in $O/prof_*.ncu-rep; do
 done
 # keep the two headline reports (C5 lcs16, C4 prevrow_cb); the rest are summarised above
 for f in $O/prof_*.ncu-rep; do
-  case $f in *c5_lcs16*|*c4_prevrow_cb*) ;; *) rm -f $f ;; esac
+  case $f in *c5_lcs16*|*c4_prevrow_hx*) ;; *) rm -f $f ;; esac
 done
 du -sh $O

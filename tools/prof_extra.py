@@ -1,7 +1,8 @@
 """One fill of each kernel that the bench line does not time, for ncu captures (development /
 measurement tool): the wavefront kernel with a TABLE output (LCS 8192²), the traceback of that
 table, the claimed-task prev-row fallback (W % 4 != 0), the Vertical twin (transpose + prev-row),
-the mInverted-L twin (mirrored inverted-L) and a batched FS fill (4 × 4096²).
+the mInverted-L twin (mirrored inverted-L), a batched FS fill (4 × 4096²) and a prev-row TABLE
+fill (prevrow_cb: the bench's prev-row lines run prevrow_hx).
 
     ncu --set full -k regex:wavefront -c 1 python tools/prof_extra.py
 """
@@ -49,6 +50,12 @@ def main():
     p5 = lddp.Plan("fs", "knight_move", m, m, lddp.OUT_TABLE, batch=B)
     p5.fill(grid=imgs, table=out)
     p5.check()
+    del imgs, out
+    gt = torch.from_numpy(inputs.gen_costs(3, n, n)).to(dev)
+    tt = torch.zeros((n, n), dtype=torch.int32, device=dev)
+    p6 = lddp.Plan("minpath3", "prev_row", n, n, lddp.OUT_SCORE | lddp.OUT_TABLE)
+    p6.fill(grid=gt, score=sc, table=tt)
+    p6.check()
     torch.cuda.synchronize()
     print("ok", int(sc.item()))
 
