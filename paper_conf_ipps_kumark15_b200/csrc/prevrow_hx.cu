@@ -429,16 +429,11 @@ static cudaError_t hx_launch(const FillParams& p, bool query, int* out, cudaStre
 template <class F>
 static cudaError_t hx_dispatch(int variant, const FillParams& p, bool query, int* out, cudaStream_t s) {
   switch (variant) {
-    case 0: return hx_launch<F, 4, 16, 96, 64, 2>(p, query, out, s);   // CW 224: 147 CTAs for C4
-    case 1: return hx_launch<F, 4, 16, 64, 64, 2>(p, query, out, s);   // CW 288
-    case 2: return hx_launch<F, 4, 16, 96, 64, 1>(p, query, out, s);   // no lane ghosts
-    case 3: return hx_launch<F, 4, 32, 64, 64, 2>(p, query, out, s);   // CW 192
-    case 4: return hx_launch<F, 4, 16, 96, 96, 2>(p, query, out, s);   // deeper ring
-    case 5: return hx_launch<F, 4, 16, 96, 32, 2>(p, query, out, s);   // shallower ring
-    case 6: return hx_launch<F, 4, 16, 64, 64, 1>(p, query, out, s);   // CW 288, no lane ghosts
-    case 7: return hx_launch<F, 4, 16, 80, 64, 1>(p, query, out, s);   // CW 256
+    // measured alternatives kept compiled; rejected ones are not built
+    case 0: return hx_launch<F, 4, 16, 96, 64, 2>(p, query, out, s);   // lane ghosts (GH = 2)
+    case 2: return hx_launch<F, 4, 16, 96, 64, 1>(p, query, out, s);   // default: CW 224, 147 CTAs for C4
+    case 6: return hx_launch<F, 4, 16, 64, 64, 1>(p, query, out, s);   // HBO 64: CW 288
     case 8: return hx_launch<F, 4, 16, 96, 32, 1>(p, query, out, s);   // 32-row ring
-    case 9: return hx_launch<F, 4, 16, 96, 96, 1>(p, query, out, s);   // 96-row ring
     default: return cudaErrorInvalidValue;
   }
 }
