@@ -135,12 +135,21 @@ __global__ void __launch_bounds__(kItWarps * 32) invl_tma_kernel(const FillParam
         ++nuse;
         if (k + kItNB - 1 < nbox) issue(k + kItNB - 1);
         const bool full = live && i0 >= ia && i0 + kItR <= ib;
+        // every lane's 32 cells inside the table and off row 0 / column 0: f reduces to
+        // max(cell, UL) + c (CellDiagMaxPlus::f without its boundary selects: two ops per cell on
+        // the chain instead of the int64 row / column tests)
+        if (__all_sync(0xffffffffu, full && i0 >= 1 && i0 + d0 + p.col0 >= 1)) {
+          const int32_t c = p.param_c;
 #pragma unroll
-        for (int u = 0; u < kItR; ++u) {
-          const int64_t i = i0 + u;
-          if (full || (live && i >= ia && i < ib)) {
-            int32_t o;
-            v = F::f(v, v, v, v, 0, 0, g[u], i, (int)(i + d) + p.col0, p.param_c, o);
+          for (int u = 0; u < kItR; ++u) v = max(g[u], v) + c;
+        } else {
+#pragma unroll
+          for (int u = 0; u < kItR; ++u) {
+            const int64_t i = i0 + u;
+            if (full || (live && i >= ia && i < ib)) {
+              int32_t o;
+              v = F::f(v, v, v, v, 0, 0, g[u], i, (int)(i + d) + p.col0, p.param_c, o);
+            }
           }
         }
       }
