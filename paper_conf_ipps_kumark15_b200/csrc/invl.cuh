@@ -76,6 +76,23 @@ __global__ void __launch_bounds__(kInvlWarps * 32) invl_kernel(const FillParams 
     load_block(cur, ibeg);
     for (int64_t i0 = ibeg; i0 < iend; i0 += BLK) {
       if (i0 + BLK < iend) load_block(nxt, i0 + BLK);
+      // whole block inside every lane's chain and short of the last row / column: no per-cell
+      // range or output tests (i, j are still passed to f: a user f may read them)
+      const bool inner = live && i0 >= ia && i0 + BLK < ib && i0 + BLK < H;
+      if (__all_sync(0xffffffffu, inner)) {
+#pragma unroll
+        for (int u = 0; u < BLK; ++u) {
+          const int64_t i = i0 + u;
+          const int64_t j = i + d;
+          typename F::OutT o;
+          v = F::f(v, v, v, v, typename F::RowCtx(0), typename F::ColCtx(0), cur[u], i,
+                   (int)j + p.col0, p.param_c, o);
+          if (TABLE) static_cast<typename F::OutT*>(p.table)[i * p.table_pitch + (MIRROR ? (int64_t)W - 1 - j : j)] = o;
+        }
+#pragma unroll
+        for (int u = 0; u < BLK; ++u) cur[u] = nxt[u];
+        continue;
+      }
 #pragma unroll
       for (int u = 0; u < BLK; ++u) {
         const int64_t i = i0 + u;
