@@ -30,7 +30,8 @@
 //  * Table edges: out-of-table cells are never forced; column 0's UL and column W-1's UR take
 //    f's boundary value (the edge warps would otherwise pace everyone through the exchange).
 //  * The last band writes last_row and the row minimum (score).
-//  * prevrow_gh_kernel (below): lane-ghost variant, measured slower, kept selectable.
+//  * Measured and rejected geometries (lane ghosts, 2-D tensor TMA, VP 8 / HB 32, 32-row rings)
+//    are no longer built (DESIGN.md §5.2 has their numbers).
 #include <cstdint>
 #include <climits>
 #include "cellfn.cuh"
@@ -523,260 +524,6 @@ __global__ void __launch_bounds__(256) prevrow_cb_kernel(const FillParams p, con
 // ---------------------------------------------------------------------------------------------
 // Compiled geometries: variant id -> (VP, HB, D); BW = 32*VP - 2*HB own columns per warp.
 // ---------------------------------------------------------------------------------------------
-// Lane-ghost variant: each lane also keeps GH ghost columns on each side (copies of its
-// neighbour lanes' own columns), refreshed by SHFL only every GH rows.  Between refreshes a row
-// needs no cross-lane exchange at all: the per-row chain shrinks from SHFL + VIMNMX3 + IADD to
-// VIMNMX3 + IADD, for (VP + 2 GH) / VP redundant cells.  Garbage from a lane window's edge
-// advances one column per row, so after GH rows the lane's own columns are still exact -- the
-// same trapezoid argument as the warp-level halo, one level down.  The cost ring rows are
-// padded by GH columns on each side so every lane reads its whole window with LDS.128.
-template <class F, int VP, int HB, int D, int GH, bool TABLE>
-__global__ void __launch_bounds__(256) prevrow_gh_kernel(const FillParams p, const __grid_constant__ CUtensorMap) {
-  using T = typename F::T;
-  using G = typename F::GridT;
-  static_assert(!(F::kMask & NB_L), "prev-row category: f must not read L");
-  static_assert(sizeof(T) == 4 && sizeof(G) == 4, "32-bit cells and costs");
-  static_assert(VP % 4 == 0 && GH % 4 == 0 && GH <= VP && HB % VP == 0 && HB % GH == 0, "geometry");
-  constexpr int EXT = 32 * VP;
-  constexpr int BW = EXT - 2 * HB;
-  constexpr int HL = HB / VP;
-  constexpr int L = VP + 2 * GH;   // lane window: [ghost GH | own VP | ghost GH]
-  constexpr int RS = EXT + 2 * GH; // padded ring row
-  static_assert(BW >= 2 * HB && L <= 32, "each edge publishes HB own columns; 32-bit masks");
-
-  extern __shared__ __align__(128) unsigned char cb_smem[];
-  const int lane = threadIdx.x & 31;
-  const int wl = threadIdx.x >> 5;
-  const int nw = blockDim.x >> 5;
-  const int q = blockIdx.x * nw + wl;
-  const int nb = p.nblocks;
-  Control* ctl = static_cast<Control*>(p.ctl);
-  const int W = p.cols;
-  const int64_t H = p.rows;
-  if (q >= nb || H <= 0) return;
-
-  G* ring = reinterpret_cast<G*>(cb_smem) + (size_t)wl * D * RS;   // [D][RS], own columns at +GH
-  const int j0 = q * BW;
-  const int e0 = j0 - HB + lane * VP;   // first own column of this lane
-  const int w0 = e0 - GH;               // first column of the lane window
-  const G* cost = static_cast<const G*>(p.grid);
-  uint32_t omask = 0;
-  T outv[L];
-#pragma unroll
-  for (int t = 0; t < L; ++t) {
-    const int col = w0 + t;
-    if (col < 0 || col >= W) omask |= 1u << t;
-    outv[t] = col < 0 ? F::left(p, 0) : F::right(p, 0);
-  }
-  const bool anyout = __any_sync(0xffffffffu, omask != 0);
-  uint32_t ssz[VP / 4];
-  const G* src[VP / 4];
-#pragma unroll
-  for (int s = 0; s < VP / 4; ++s) {
-    const int col = e0 + 4 * s;
-    const bool in = col >= 0 && col < W;
-    ssz[s] = in ? 16u : 0u;
-    asm volatile("mov.b32 %0, %0;" : "+r"(ssz[s]));
-    src[s] = cost + (in ? col : 0);
-  }
-  int64_t pitch = p.grid_pitch;
-  asm volatile("mov.b64 %0, %0;" : "+l"(pitch));
-  const uint32_t rbase = smem_u32(ring);
-  const uint32_t ibeg = rbase + (GH + lane * VP) * 4, iend = ibeg + (D - 1) * RS * 4;
-  uint32_t idst = ibeg;
-  int ileft = (int)H;
-  int64_t ioff = 0;
-  for (int k = 0; k < D - 1; ++k) {
-    if (ileft > 0) {
-#pragma unroll
-      for (int s = 0; s < VP / 4; ++s) cb_cp16s(idst + 16 * s, src[s] + ioff, ssz[s]);
-    }
-    ioff += pitch;
-    --ileft;
-    idst += RS * 4;
-    cp_async_commit();
-  }
-  cp_async_wait_group<D - 2>();
-  __syncwarp();
-  auto load_row = [&](int slot, G (&g)[L]) {
-    const G* gs = ring + slot * RS + lane * VP;   // = padded window start (own - GH)
-#pragma unroll
-    for (int s = 0; s < L / 4; ++s) {
-      const int4 t = *reinterpret_cast<const int4*>(gs + 4 * s);
-      g[4 * s] = t.x; g[4 * s + 1] = t.y; g[4 * s + 2] = t.z; g[4 * s + 3] = t.w;
-    }
-  };
-  G g[L];
-  load_row(0, g);
-  int cslot = 0;
-
-  T cur[L];
-#pragma unroll
-  for (int t = 0; t < L; ++t) cur[t] = ((omask >> t) & 1u) ? outv[t] : F::top(p, w0 + t);
-
-  auto refresh = [&]() {   // ghosts <- the neighbour lanes' own edge columns
-#pragma unroll
-    for (int t = 0; t < GH; ++t) {
-      const T lg = __shfl_up_sync(0xffffffffu, cur[VP + t], 1);        // lane-1's own [VP-GH, VP)
-      const T rg = __shfl_down_sync(0xffffffffu, cur[GH + t], 1);      // lane+1's own [0, GH)
-      cur[t] = ((omask >> t) & 1u) ? outv[t] : lg;
-      cur[GH + VP + t] = ((omask >> (GH + VP + t)) & 1u) ? outv[GH + VP + t] : rg;
-    }
-  };
-
-  // edge-pair tags: fill epoch (mod 4096) and band + 1 in disjoint bit fields -- every slot a fill
-  // uses is rewritten by it, so a pair left by an earlier fill of this workspace never matches
-  const uint32_t tag0 = (uint32_t)(p.epoch & 0x7FFu) << 20;
-  uint64_t* edges = reinterpret_cast<uint64_t*>(p.bnd);
-  const bool lhalo = lane < HL, rhalo = lane >= 32 - HL;
-  const bool ledge = lane >= HL && lane < 2 * HL;
-  const bool redge = lane >= 32 - 2 * HL && lane < 32 - HL;
-
-  auto band = [&](const int nr, const int64_t r0, auto out_tag) {
-    constexpr bool OUT = decltype(out_tag)::value;
-#pragma unroll 1
-    for (int r = 0; r < nr; ++r) {
-      if (ileft > 0) {
-#pragma unroll
-        for (int s = 0; s < VP / 4; ++s) cb_cp16s(idst + 16 * s, src[s] + ioff, ssz[s]);
-      }
-      ioff += pitch;
-      --ileft;
-      idst = (idst == iend) ? ibeg : idst + RS * 4;
-      cp_async_commit();
-      cp_async_wait_group<D - 2>();
-      cslot = (cslot + 1 == D) ? 0 : cslot + 1;
-      G gn[L];
-      load_row(cslot, gn);
-      const int64_t row = r0 + r;
-      T nw_[L];
-#pragma unroll
-      for (int t = 0; t < L; ++t) {
-        const T UL = (t > 0) ? cur[t - 1] : cur[0];        // window edges: garbage, absorbed
-        const T UR = (t < L - 1) ? cur[t + 1] : cur[L - 1];
-        typename F::OutT o;
-        T x = F::f(cur[t], UL, cur[t], UR, typename F::RowCtx(0), typename F::ColCtx(0), g[t], row, w0 + t,
-                   p.param_c, o);
-        if (OUT) x = ((omask >> t) & 1u) ? outv[t] : x;
-        nw_[t] = x;
-        if (TABLE && t >= GH && t < GH + VP) {
-          const int col = w0 + t;
-          if (col >= j0 && col < j0 + BW && col < p.cols)
-            static_cast<typename F::OutT*>(p.table)[row * p.table_pitch + col] = o;
-        }
-      }
-#pragma unroll
-      for (int t = 0; t < L; ++t) {
-        cur[t] = nw_[t];
-        g[t] = gn[t];
-      }
-      if ((r + 1) % GH == 0) refresh();
-    }
-  };
-
-#pragma unroll 1
-  for (int64_t r0 = 0; r0 < H; r0 += HB) {
-    const int nr = (int)((H - r0 < HB) ? (H - r0) : HB);
-    if (anyout) band(nr, r0, std::true_type{});
-    else band(nr, r0, std::false_type{});
-    if (r0 + HB >= H) break;
-    const int bnd_ = (int)(r0 / HB);
-    const uint32_t tag = tag0 | (((uint32_t)bnd_ + 1u) & 0xFFFFFu);
-    uint64_t* mine = edges + ((size_t)q * 4 + (bnd_ & 3)) * 2 * HB;
-    if (ledge || redge) {
-      uint64_t* d = mine + (ledge ? 0 : HB) + (ledge ? (lane - HL) : (lane - (32 - 2 * HL))) * VP;
-#pragma unroll
-      for (int v = 0; v < VP; v += 2)
-        cb_st_pair2(d + v, ((uint64_t)tag << 32) | (uint32_t)cur[GH + v], ((uint64_t)tag << 32) | (uint32_t)cur[GH + v + 1]);
-    }
-    const int nbq = lhalo ? q - 1 : q + 1;
-    const bool need = (lhalo && q > 0) || (rhalo && q + 1 < nb);
-    const uint64_t* sp = nullptr;
-    if (need) sp = edges + ((size_t)nbq * 4 + (bnd_ & 3)) * 2 * HB + (lhalo ? HB + lane * VP : (lane - (32 - HL)) * VP);
-    uint64_t pr[VP];
-    bool ok = true;
-    if (need) {
-#pragma unroll
-      for (int v = 0; v < VP; v += 2) cb_ld_pair2(sp + v, pr[v], pr[v + 1]);
-#pragma unroll
-      for (int v = 0; v < VP; ++v) ok = ok && ((uint32_t)(pr[v] >> 32) == tag);
-    }
-    if (!__all_sync(0xffffffffu, ok)) {
-      Backoff bo;
-      int spins = 0;
-      while (true) {
-        if (!ok) {
-          ok = true;
-#pragma unroll
-          for (int v = 0; v < VP; v += 2) cb_ld_pair2(sp + v, pr[v], pr[v + 1]);
-#pragma unroll
-          for (int v = 0; v < VP; ++v) ok = ok && ((uint32_t)(pr[v] >> 32) == tag);
-        }
-        if (__all_sync(0xffffffffu, ok)) break;
-        if (++spins > 64 && !bo.tick(ctl, p.timeout_ns)) return;
-      }
-    }
-    if (need) {
-#pragma unroll
-      for (int v = 0; v < VP; ++v) cur[GH + v] = (T)(uint32_t)pr[v];
-    }
-    refresh();   // ghosts of the replaced halo lanes and of their neighbours
-  }
-  cp_async_wait_group<0>();
-
-  T mn = INT_MAX;
-#pragma unroll
-  for (int v = 0; v < VP; ++v) {
-    const int col = e0 + v;
-    if (col >= j0 && col < j0 + BW && col < W) {
-      if (p.last_row != nullptr) static_cast<T*>(p.last_row)[col] = cur[GH + v];
-      mn = min(mn, cur[GH + v]);
-    }
-  }
-  if (F::kScore == SCORE_ROW_MIN && p.score != nullptr) {
-    unsigned* rowmin_done = &ctl->pad[0];
-    T* rowmins = reinterpret_cast<T*>(p.prog);
-#pragma unroll
-    for (int off = 16; off > 0; off >>= 1) mn = min(mn, __shfl_xor_sync(0xffffffffu, mn, off));
-    if (lane == 0) {
-      rowmins[q] = mn;
-      __threadfence();
-      const unsigned d = atomicAdd(rowmin_done, 1u);
-      if (d == (unsigned)nb - 1) {
-        __threadfence();
-        T best = INT_MAX;
-        for (int k = 0; k < nb; ++k) best = min(best, __ldcg(rowmins + k));
-        *static_cast<T*>(p.score) = best;
-        atomicExch(rowmin_done, 0u);
-      }
-    }
-  }
-}
-
-template <class F, int VP, int HB, int D, int GH>
-static cudaError_t gh_launch(const FillParams& p, int nw, bool query, int* out, cudaStream_t s) {
-  const size_t smem = (size_t)nw * D * (32 * VP + 2 * GH) * sizeof(typename F::GridT);
-  auto kt = prevrow_gh_kernel<F, VP, HB, D, GH, true>;
-  auto kf = prevrow_gh_kernel<F, VP, HB, D, GH, false>;
-  cudaError_t e = cudaFuncSetAttribute(kt, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  if (e == cudaSuccess) e = cudaFuncSetAttribute(kf, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  if (e != cudaSuccess) return e;
-  auto k = p.table != nullptr ? kt : kf;
-  if (query) {
-    int occ = 0;
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k, nw * 32, smem);
-    out[0] = 32 * VP - 2 * HB;
-    out[1] = occ;
-    return e;
-  }
-  CUtensorMap tm;
-  memset(&tm, 0, sizeof(tm));
-  const int grid = (p.nblocks + nw - 1) / nw;
-  FillParams pp = p;
-  void* args[] = {&pp, &tm};
-  return cudaLaunchCooperativeKernel((const void*)k, dim3(grid), dim3(nw * 32), args, smem, s);
-}
-
 // cuTensorMapEncodeTiled through the runtime's driver entry point (no libcuda link needed).
 static PFN_cuTensorMapEncodeTiled_v12000 cb_encode_fn() {
   static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
@@ -831,13 +578,9 @@ template <class F>
 static cudaError_t cb_dispatch(int variant, const FillParams& p, int nw, bool query, int* out, cudaStream_t s) {
   switch (variant) {
     case 0: return cb_launch<F, 8, 64, 48>(p, nw, query, out, s);   // BW 128
-    case 1: return cb_launch<F, 8, 32, 48>(p, nw, query, out, s);
     case 5: return cb_launch<F, 4, 32, 64>(p, nw, query, out, s);   // BW 64
-    case 8: return cb_launch<F, 4, 32, 96, 2>(p, nw, query, out, s);   // BW 64, 2-D tensor TMA, 32-row groups
-    case 10: return gh_launch<F, 4, 32, 64, 4>(p, nw, query, out, s);  // BW 64, lane ghosts: SHFL every 4 rows
     case 13: return cb_launch<F, 2, 16, 64>(p, nw, query, out, s);      // BW 32, 8-byte segments, 1024 warps for C4
     case 17: return cb_launch<F, 6, 48, 48>(p, nw, query, out, s);      // BW 96, exchange every 48 rows
-    case 18: return cb_launch<F, 6, 48, 32>(p, nw, query, out, s);      // BW 96, 32-row ring
     default: return cudaErrorInvalidValue;
   }
 }

@@ -37,7 +37,7 @@ def cb_env():
             os.environ[k] = v
 
 
-@pytest.mark.parametrize("variant,warps", [(0, 2), (1, 1), (0, 4), (5, 4), (5, 2), (8, 2), (8, 1), (8, 4), (10, 2), (10, 1), (10, 4), (13, 2), (13, 4), (13, 8), (17, 4), (17, 2), (18, 4)])
+@pytest.mark.parametrize("variant,warps", [(0, 2), (0, 1), (0, 4), (5, 4), (5, 2), (5, 1), (13, 2), (13, 4), (13, 8), (17, 4), (17, 2)])
 @pytest.mark.parametrize("shape", CB_SHAPES)
 def test_minpath3_cb(cb_env, variant, warps, shape):
     cb_env(variant, warps)
@@ -47,7 +47,7 @@ def test_minpath3_cb(cb_env, variant, warps, shape):
     outs = ("score", "last_row", "table") if ref.table is not None else ("score", "last_row")
     got = run_gpu("minpath3", "prev_row", grid=c, outputs=outs, reps=2)
     info = json.loads(got["plan"])
-    assert info["kernel"] == "prevrow_cb", info   # (variants 10-12: the lane-ghost kernel, same plan kind)
+    assert info["kernel"] == "prevrow_cb", info
     assert info["variant"] == variant
     np.testing.assert_array_equal(got["last_row"], ref.last_row)
     assert got["score"] == ref.score
@@ -55,7 +55,7 @@ def test_minpath3_cb(cb_env, variant, warps, shape):
         np.testing.assert_array_equal(got["table"], ref.table)
 
 
-@pytest.mark.parametrize("variant", [0, 1, 5, 8, 10, 13])
+@pytest.mark.parametrize("variant", [0, 5, 13, 17])
 @pytest.mark.parametrize("shape", [(1000, 1000), (300, 2052)])
 def test_min2plus_diagmaxplus_cb(cb_env, variant, shape):
     cb_env(variant, 2)
