@@ -589,7 +589,9 @@ lddp_status lddp_plan(const lddp_desc* desc, lddp_plan_t* out) {
     if (d.category == LDDP_CAT_ANTI_DIAGONAL && d.func == LDDP_F_LCS && !table && !force_wf && !force_ad) {
       // packed 16x2 LCS kernel (lcs16.cu): P row pairs per lane, lane lag E
       pl->kind = 4;
-      pl->R = d.tile_rows > 0 ? (d.tile_rows + 1) / 2 : env_int("LDDP_L16_P", 6);
+      // default P (measured on one B200): 6 (384-row strips) for C5-sized tables; 4 for tables of
+      // <= 4096 rows, where pipeline fill / drain over few strips dominates (C1 0.065 -> 0.051 ms)
+      pl->R = d.tile_rows > 0 ? (d.tile_rows + 1) / 2 : env_int("LDDP_L16_P", d.rows <= 4096 ? 4 : 6);
       pl->E = env_int("LDDP_L16_E", 2);
       pl->W = 1;
       pl->SIG = 0;
