@@ -109,3 +109,14 @@ def test_hx_full_width_c4_sample(hx_env):
     assert info["kernel"] == "prevrow_hx" and info["grid"] == 147
     np.testing.assert_array_equal(got["last_row"], ref.last_row)
     assert got["score"] == ref.score
+
+
+def test_hx_too_wide_falls_back(hx_env):
+    """More CTAs than can be co-resident (W > 148 x 224 columns): the plan keeps prevrow_cb."""
+    hx_env(2)
+    c = inputs.gen_costs(6, 40, 40000)
+    ref = oracle.minpath3(c)
+    got = run_gpu("minpath3", "prev_row", grid=c, outputs=("score", "last_row"))
+    assert json.loads(got["plan"])["kernel"] != "prevrow_hx"
+    np.testing.assert_array_equal(got["last_row"], ref.last_row)
+    assert got["score"] == ref.score
