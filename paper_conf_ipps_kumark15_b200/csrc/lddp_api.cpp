@@ -688,7 +688,10 @@ lddp_status lddp_plan(const lddp_desc* desc, lddp_plan_t* out) {
         else if (rows == 2) variant = 2;
         else if (rows == 8) variant = 3;
         else variant = 0;
-        if (table) variant = 0;   // TABLE mode is compiled for the default variant only
+        // TABLE mode is compiled for variants 2 (R2, skewed: measured ~10 % faster for LCS /
+        // Levenshtein / DTW 8192^2 TABLE fills, tools/table_time.py) and 0 (R4)
+        if (table && variant != 0) variant = 2;
+        if (table && v_env == 0) variant = 0;
       }
       if (d.tile_warps != 0 && d.tile_warps != kWfWarps) {
         delete pl;

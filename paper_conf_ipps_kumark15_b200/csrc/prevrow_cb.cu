@@ -410,7 +410,11 @@ __global__ void __launch_bounds__(256) prevrow_cb_kernel(const FillParams p, con
     for (int64_t r0 = 0; r0 < H; r0 += HB) {
       const int nr = (int)((H - r0 < HB) ? (H - r0) : HB);
       // development trace (LDDP_TRACE): per band of block `trace_chunks`, clock64 at entry / exit
+#ifdef LDDP_CB_TRACE
       const bool trc = p.trace != nullptr && q == p.trace_chunks && lane == 0 && r0 / HB < 4096;
+#else
+      constexpr bool trc = false;   // the per-band checks cost ~8 % (measured on prevrow_hx)
+#endif
       const long long tb0 = trc ? clock64() : 0;
       if (anyout)
         cb_band<F, VP, D, TABLE, true, MODE>(bk, tmap, lane, p, cur, g, nr, r0, ring, cslot, idst, ileft, ioff, pitch, src, ssz, ed, e0, j0, BW);

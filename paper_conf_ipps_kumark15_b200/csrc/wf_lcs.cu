@@ -4,6 +4,7 @@ namespace lddp {
 int wf_dispatch_lcs(int op, int variant, bool table, const FillParams* p, int grid, cudaStream_t s) {
   LDDP_WF_CASE(CellLCS, WF_A_R4_S0, 4, 0, 2, false)
   LDDP_WF_CASE(CellLCS, WF_A_R2_S1, 2, 1, 1, false)
+  LDDP_WF_CASE(CellLCS, WF_A_R2_S1, 2, 1, 1, true)
   LDDP_WF_CASE(CellLCS, WF_A_R8_S1, 8, 1, 1, false)
   LDDP_WF_CASE(CellLCS, WF_A_R4_S0, 4, 0, 2, true)
   LDDP_WF_CASE(CellLCS, WF_K_R1, 1, 2, 2, false)

@@ -2,6 +2,9 @@
 including the halo exchange.  Development tool.
 
     python tools/cb_trace.py --H 32768 --W 32768 --block 100
+
+Needs a trace build: make -C paper_conf_ipps_kumark15_b200 -B EXTRA=-DLDDP_CB_TRACE (the per-band
+trace checks are compiled out of the product build).
 """
 import argparse
 import json

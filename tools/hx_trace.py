@@ -3,6 +3,9 @@ cycles per inner band of rows and per band including the exchange; optional LDDP
 switches (1 = no outer L2 waits, 2 = no inner barrier, wrong results).  Development tool.
 
     python tools/hx_trace.py --cta 70 --debug 0 1 2 3
+
+Needs a trace build: make -C paper_conf_ipps_kumark15_b200 -B EXTRA=-DLDDP_HX_TRACE (the per-band
+trace checks are compiled out of the product build).
 """
 import argparse
 import json
