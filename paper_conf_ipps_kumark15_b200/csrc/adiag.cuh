@@ -108,8 +108,13 @@ __device__ __forceinline__ uint64_t ad_pair(uint32_t bits, uint32_t tag) {
 // S = 1 ("split"): the lane's rows [R/2, R) run one column behind rows [0, R/2) -- their U at
 // column c-1 is the upper half's value from the previous step -- so a step holds two independent
 // chains of R/2 cells (ILP 2) for one extra step of lane lag (ELAG = E + S).
-template <class F, int R, int W, int E, int S = 0>
+template <class F, int R, int W, int E, int S = 0, bool TB = false>
 struct AdWarp {
+  // TB: TABLE output -- every cell of the strip goes to the row-major table.  A lane's R values
+  // per step are staged in a per-warp shared tile [R][32 lanes][33] (conflict-free both ways); at
+  // the end of each chunk the warp writes the tile row by row, 32 consecutive columns per store
+  // (coalesced), skipping virtual rows and columns outside [0, n).
+  static_assert(!TB || !S, "TABLE output: unsplit geometries");
   static constexpr int ELAG = E + S;   // lane-to-lane column lag
   // strip-boundary pairs loaded half a chunk ahead inside the group loop: DTW (fully unrolled
   // groups) and one-warp CTAs (every warp reads its top row from global memory); for 4-warp
@@ -146,6 +151,7 @@ struct AdWarp {
                     // ring holds codes and a step's mask is one PRMT of mpk (no table lookup)
   int32_t one;      // run-time 1 held in a register (opaque to ptxas: no per-use constant loads)
   int64_t irow0;    // global row of this lane's row 0
+  uint32_t* tbl;    // TB: this warp's staging tile (32 * R * 33 words)
 
   // ---- per-warp handoff state
   uint64_t tp;      // this lane's top pair of the current chunk (column 32k + lane)
@@ -383,6 +389,7 @@ struct AdWarp {
             UL = hist[r];
             U = v;
             nw[r] = v;
+            if constexpr (TB) tbl[(r * 32 + lane) * 33 + 8 * g + u] = ad_bits(v);
           }
         }
         bv[u] = nw[R - 1];
@@ -406,6 +413,46 @@ struct AdWarp {
         d[1] = make_uint4(ad_bits(bv[4]), ad_bits(bv[5]), ad_bits(bv[6]), ad_bits(bv[7]));
       }
     }
+    if constexpr (TB) store_tile(p, lane, k);
+  }
+
+  // TB: the chunk's tile -> table.  Row r of lane src holds columns 32k - E - src * ELAG + su at
+  // tile [(r * 32 + src) * 33 + su]; lane su of the warp stores that column (one coalesced row
+  // segment per (src, r)).
+  __device__ __forceinline__ void store_tile(const FillParams& p, const int lane, const int k) {
+    __syncwarp();
+    const int n = p.cols;
+    const int64_t m = p.rows;
+    const int64_t wtop = irow0 - (int64_t)lane * R;
+    const int64_t pitch = p.table_pitch;
+    // this lane's column for src = 0 and the pointer of (src = 0, r = 0); src + 1 is R rows down
+    // and ELAG columns left
+    const int col0 = 32 * k - E + lane;
+    uint32_t* rowp = static_cast<uint32_t*>(p.table) + wtop * pitch + col0;
+    const int64_t step_src = (int64_t)R * pitch - ELAG;
+    const bool fast = (32 * k - E - 31 * ELAG >= 0) && (32 * k - E + 31 < n) && wtop >= 0 && wtop + 32 * R <= m;
+    if (__all_sync(0xffffffffu, fast)) {   // every (row, column) of the tile inside the table
+#pragma unroll 4
+      for (int src = 0; src < 32; ++src) {
+#pragma unroll
+        for (int r = 0; r < R; ++r) rowp[r * pitch] = tbl[(r * 32 + src) * 33 + lane];
+        rowp += step_src;
+      }
+    } else {
+#pragma unroll 4
+      for (int src = 0; src < 32; ++src) {
+        const int col = col0 - src * ELAG;
+        const bool cin = (unsigned)col < (unsigned)n;
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+          const int64_t row = wtop + (int64_t)src * R + r;
+          const uint32_t v = tbl[(r * 32 + src) * 33 + lane];
+          if (cin && row >= 0 && row < m) rowp[r * pitch] = v;
+        }
+        rowp += step_src;
+      }
+    }
+    __syncwarp();
   }
 
   template <bool CHECKED, bool SM>
@@ -441,9 +488,12 @@ struct AdWarp {
   }
 };
 
-template <class F, int R, int W, int E, int S = 0>
+template <class F, int R, int W, int E, int S = 0, bool TB = false>
 __global__ void __launch_bounds__(W * 32, 1) adiag_kernel(const FillParams p) {
-  using AW = AdWarp<F, R, W, E, S>;
+  using AW = AdWarp<F, R, W, E, S, TB>;
+  static_assert(!TB || W == 1, "TABLE output: one-warp strips");
+  static_assert(!TB || sizeof(typename F::OutT) == 4, "TABLE output: 32-bit cells");
+  __shared__ uint32_t tbl_sh[TB ? W : 1][TB ? 32 * R * 33 : 1];   // TB staging tiles
   using T = typename AW::T;
   constexpr int SH = AW::SH;
   __shared__ __align__(16) uint64_t ring[W][kAdRing][32];   // ring[w]: top stream of warp w >= 1
@@ -509,6 +559,7 @@ __global__ void __launch_bounds__(W * 32, 1) adiag_kernel(const FillParams p) {
       if (threadIdx.x == 0 && ok) window_consume_ack(p, s);
     }
     aw.cring = cring[wid];
+    aw.tbl = tbl_sh[TB ? wid : 0];
     aw.one = ad_ld_smem_i32(&one_sh);   // a volatile load: ptxas cannot rematerialise it per use
     aw.small = false;
     if constexpr (F::kMatchCells) {

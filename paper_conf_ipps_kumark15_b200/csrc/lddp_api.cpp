@@ -133,12 +133,18 @@ int wf_dispatch(int func, int op, int variant, bool table, const FillParams* p, 
 
 // Compiled adiag geometries (tools/gen_adiag.py): f, rows per lane R, lane lag E, warps per CTA W.
 struct AdGeom {
-  int func, R, E, W, S;
+  int func, R, E, W, S, TB;   // TB: TABLE output (one-warp strips, staging tile)
   cudaError_t (*launch)(const FillParams&, int, cudaStream_t);
 };
 const AdGeom kAdGeoms[] = {
 LDDP_AD_TABLE_ROWS
 };
+
+bool ad_has_table(int func) {
+  for (const auto& g : kAdGeoms)
+    if (g.func == func && g.TB) return true;
+  return false;
+}
 
 // Lane-systolic anti-diagonal geometry model, constants from the B200
 // microbenchmarks in tools/micro (ad_step2.cu, lat.cu).  One warp's step (R cells per lane)
@@ -623,7 +629,8 @@ lddp_status lddp_plan(const lddp_desc* desc, lddp_plan_t* out) {
       const int64_t fb_strips = (d.rows + 191) / 192;
       pl->ws_bytes = pl->off_bnd + (size_t)std::max<int64_t>(std::max(pl->nstrips, (int)fb_strips) - 1, 1) *
                                        pl->bnd_stride * 8;
-    } else if (d.category == LDDP_CAT_ANTI_DIAGONAL && seq_func(d.func) && !table && !force_wf) {
+    } else if (d.category == LDDP_CAT_ANTI_DIAGONAL && seq_func(d.func) && !force_wf &&
+               (!table || ad_has_table(d.func))) {
       // lane-systolic anti-diagonal kernel (adiag.cuh)
       pl->kind = 3;
       int Rq = d.tile_rows > 0 ? d.tile_rows : env_int("LDDP_AD_R", 0);
@@ -649,6 +656,7 @@ lddp_status lddp_plan(const lddp_desc* desc, lddp_plan_t* out) {
         if (Wq > 0 && g.W != Wq) continue;
         if (Sq >= 0 && g.S != Sq) continue;
         if (Sq < 0 && g.S) continue;   // split geometries only on request: measured slower on B200 (C5 6.9 -> 11.6 ms)
+        if (g.TB != (table ? 1 : 0)) continue;   // TABLE fills: the staging-tile instantiations
         double c = ad_cost(d.func, g.R, g.E, g.W, g.S, d.rows, std::max<int64_t>(d.cols, 1), pl->sms);
         if (Rq > 0) c += 1e200 * std::abs(g.R - Rq);   // nearest compiled R to the request
         if (getenv("LDDP_PLAN_DEBUG"))

@@ -149,6 +149,8 @@ def test_plan_describe_and_workspace(L):
     plan = L.lddp_plan(d)
     try:
         import json
-        assert json.loads(L.lddp_plan_describe(plan))["kernel"] == "wavefront"   # TABLE output
+        # TABLE output: the adiag kernel's staging-tile instantiation (one-warp strips)
+        info = json.loads(L.lddp_plan_describe(plan))
+        assert info["kernel"] == "adiag" and info["warps"] == 1, info
     finally:
         L.lddp_plan_destroy(plan)

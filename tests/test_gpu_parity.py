@@ -4,6 +4,8 @@ and chunk sizes +-1, ragged strips / bands).  Integer f's and FS must be bit-exa
 expected bit-exact (same per-cell operation sequence) and is held to <= 1e-5 relative, the north
 star's tolerance.  Schedule independence: the same f under every covering category gives the
 identical table."""
+import json
+
 import numpy as np
 import pytest
 
@@ -187,3 +189,26 @@ def test_small_grid_forces_strip_reuse():
     got = run_gpu("minpath3", "prev_row", grid=c, outputs=("score", "last_row"), grid_ctas=1)
     assert got["score"] == r.score
     np.testing.assert_array_equal(got["last_row"], r.last_row)
+
+
+@pytest.mark.parametrize("func", ["lcs", "levenshtein", "dtw"])
+@pytest.mark.parametrize("shape", [(1, 1), (1, 300), (300, 1), (127, 33), (128, 64), (129, 95), (385, 1000),
+                                   (1000, 777), (2000, 2049)])
+@pytest.mark.parametrize("kernel", ["default", "wavefront"])
+def test_table_fill_kernels(func, shape, kernel, monkeypatch):
+    """TABLE fills of the anti-diagonal sequence f's: the adiag staging-tile kernel (default) and
+    the wavefront kernel (LDDP_KERNEL=wavefront) both equal the oracle's table element by element
+    (bit-exact for LCS / Levenshtein; DTW too: same fp32 operation order)."""
+    if kernel == "wavefront":
+        monkeypatch.setenv("LDDP_KERNEL", "wavefront")
+    m, n = shape
+    if func == "dtw":
+        a, b = inputs.gen_walks(7 * m + n, m, n)
+        ref = oracle.dtw(a, b, table=True)
+    else:
+        a, b = inputs.gen_strings(7 * m + n, m, n)
+        ref = getattr(oracle, func)(a, b, table=True)
+    got = run_gpu(func, "anti_diagonal", a=a, b=b, outputs=("score", "table"))
+    assert json.loads(got["plan"])["kernel"] == ("wavefront" if kernel == "wavefront" else "adiag")
+    np.testing.assert_array_equal(got["table"], ref.table)
+    assert got["score"] == ref.score

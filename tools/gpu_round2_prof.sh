@@ -22,6 +22,7 @@ cap c6_invl invl python bench.py --workload C6 --no-others --no-cpu --steps 1 --
 cap c7_prevrow_hx prevrow_hx python bench.py --workload C7 --no-others --no-cpu --steps 1 --warmup 3
 cap c8_fsk_batch fsk python bench.py --workload C8 --no-others --no-cpu --steps 1 --warmup 3
 SKIP=0 cap x_wavefront_table wavefront python tools/prof_extra.py
+SKIP=0 cap x_adiag_table adiag python tools/prof_extra.py
 SKIP=0 cap x_traceback traceback python tools/prof_extra.py
 SKIP=0 cap x_prevrow_fallback "prevrow_kernel" python tools/prof_extra.py
 SKIP=0 cap x_transpose transpose python tools/prof_extra.py

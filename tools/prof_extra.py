@@ -1,6 +1,6 @@
 """One fill of each kernel that the bench line does not time, for ncu captures (development /
-measurement tool): the wavefront kernel with a TABLE output (LCS 8192²), the traceback of that
-table, the claimed-task prev-row fallback (W % 4 != 0), the Vertical twin (transpose + prev-row),
+measurement tool): LCS 8192² TABLE fills on the adiag staging-tile kernel and on the wavefront
+kernel, the traceback of that table, the claimed-task prev-row fallback (W % 4 != 0), the Vertical twin (transpose + prev-row),
 the mInverted-L twin (mirrored inverted-L), a batched FS fill (4 × 4096²) and a prev-row TABLE
 fill (prevrow_cb: the bench's prev-row lines run prevrow_hx).
 
@@ -24,9 +24,14 @@ def main():
     ta, tb = torch.from_numpy(a).to(dev), torch.from_numpy(b).to(dev)
     tab = torch.zeros((n, n), dtype=torch.int32, device=dev)
     sc = torch.zeros(1, dtype=torch.int32, device=dev)
-    plan = lddp.Plan("lcs", "anti_diagonal", n, n, lddp.OUT_SCORE | lddp.OUT_TABLE)
+    plan = lddp.Plan("lcs", "anti_diagonal", n, n, lddp.OUT_SCORE | lddp.OUT_TABLE)   # adiag, TABLE tile
     plan.fill(a=ta, b=tb, score=sc, table=tab)
     plan.check()
+    os.environ["LDDP_KERNEL"] = "wavefront"   # the generic wavefront kernel on the same TABLE fill
+    pw = lddp.Plan("lcs", "anti_diagonal", n, n, lddp.OUT_SCORE | lddp.OUT_TABLE)
+    del os.environ["LDDP_KERNEL"]
+    pw.fill(a=ta, b=tb, score=sc, table=tab)
+    pw.check()
     pi, pj = plan.traceback(ta, tb, tab)
     torch.cuda.synchronize()
     del tab

@@ -33,7 +33,16 @@ def main():
             a, b = torch.from_numpy(x).to(dev), torch.from_numpy(y).to(dev)
             dt = torch.int32
         ref = torch.zeros(1, dtype=dt, device=dev)
-        lddp.Plan(func, "anti_diagonal", n, n, lddp.OUT_SCORE).fill(a=a, b=b, score=ref)
+        p0 = lddp.Plan(func, "anti_diagonal", n, n, lddp.OUT_SCORE)
+        p0.fill(a=a, b=b, score=ref)
+        s0, e0 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        s0.record()
+        for _ in range(5):
+            p0.fill(a=a, b=b, score=ref)
+        e0.record()
+        torch.cuda.synchronize()
+        print(json.dumps({"func": func, "n": n, "score_only_ms": round(s0.elapsed_time(e0) / 5, 3),
+                          "kernel": json.loads(p0.info)["kernel"]}), flush=True)
         for v in args.variant:
             os.environ["LDDP_WF_VARIANT"] = str(v)
             tab = torch.zeros((n, n), dtype=dt, device=dev)
