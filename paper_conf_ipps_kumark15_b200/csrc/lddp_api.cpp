@@ -698,8 +698,10 @@ lddp_status lddp_plan(const lddp_desc* desc, lddp_plan_t* out) {
         else variant = 0;
         // TABLE mode is compiled for variants 2 (R2, skewed: measured ~10 % faster for LCS /
         // Levenshtein / DTW 8192^2 TABLE fills, tools/table_time.py) and 0 (R4)
-        if (table && variant != 0) variant = 2;
-        if (table && v_env == 0) variant = 0;
+        if (table) {
+          variant = (v_env == 0) ? 0 : 2;
+          if (wf_dispatch(d.func, 2, variant, true, nullptr, 0, nullptr) < 0) variant = 0;   // R2 TABLE: seq f's only
+        }
       }
       if (d.tile_warps != 0 && d.tile_warps != kWfWarps) {
         delete pl;
