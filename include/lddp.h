@@ -141,8 +141,11 @@ typedef struct {
     int32_t tile_rows;       /* tuning: rows per lane (anti-diagonal / knight), 0 = auto        */
     int32_t tile_warps;      /* tuning: compute warps per CTA, 0 = auto                         */
     int32_t band_rows;       /* tuning, prev-row category: trapezoid band height HB (rows between
-                                two halo exchanges of the column-block kernel): 16, 32, 48 or
-                                64 (else LDDP_ERR_UNSUPPORTED); 0 = auto (32)                    */
+                                two halo exchanges of the column-block kernel prevrow_cb): 16,
+                                32, 48 or 64 (else LDDP_ERR_UNSUPPORTED); 0 = auto (SCORE /
+                                LAST_ROW fills on one GPU: the hierarchical-exchange kernel,
+                                inner halos every 16 rows, CTA-edge halos every 96; TABLE
+                                fills and lddp_fill_multi: prevrow_cb with HB = 32)           */
     int32_t grid_ctas;       /* tuning: persistent grid size, 0 = auto (SMs x occupancy)        */
     int32_t batch;           /* FS_DITHER only: number of independent images stacked along the
                                 rows (image b = rows [b*rows, (b+1)*rows) of inputs.grid and of
@@ -164,9 +167,10 @@ typedef struct {
                                 per fill, fall back to the generic kernels otherwise:
                                 - FS (fsk.cu): cols % 16 == 0, grid and table pitches multiples
                                   of 16 bytes, 16-byte aligned bases;
-                                - prev-row (prevrow_cb.cu): 32-bit grid, cols % 4 == 0, pitch
-                                  % 4 == 0, 16-byte aligned base, and the column blocks
-                                  co-resident on the device (checked at plan time)          */
+                                - prev-row (prevrow_hx.cu / prevrow_cb.cu): 32-bit grid,
+                                  cols % 4 == 0, pitch % 4 == 0, 16-byte aligned base, and the
+                                  column blocks co-resident on the device (checked at plan
+                                  time; prevrow_hx also rows < 2^30, pitch < 2^29)           */
 } lddp_inputs;
 
 typedef struct {
