@@ -429,8 +429,10 @@ lddp_status launch(lddp_plan_t pl, const FillParams& p, cudaStream_t s) {
     q.strip_rows = 192;
     q.bnd_stride = (int64_t)std::max((q.cols + 31) / 32, 1) * 32;
     e = lddp::ad_lcs_r6e2w1(q, std::min(q.nstrips, pl->sms * 8), s);
-  } else if (pl->kind == 1 && pl->hx_variant >= 0 && p.table == nullptr && p.grid_pitch % 4 == 0 &&
-             p.grid_pitch < ((int64_t)1 << 29) && ((reinterpret_cast<uintptr_t>(p.grid) & 15) == 0)) {
+  } else if (pl->kind == 1 && pl->hx_variant >= 0 && p.grid_pitch % 4 == 0 && p.grid_pitch < ((int64_t)1 << 29) &&
+             ((reinterpret_cast<uintptr_t>(p.grid) & 15) == 0) &&
+             (p.table == nullptr || (p.table_pitch % 4 == 0 && p.table_pitch < ((int64_t)1 << 29) &&
+                                     (reinterpret_cast<uintptr_t>(p.table) & 15) == 0))) {
     int dummy[3];
     e = lddp::launch_prevrow_hx(pl->desc.func, pl->hx_variant, p, false, dummy, s);
   } else if (pl->kind == 1 && pl->cb_variant >= 0 && (p.grid_pitch % 4 == 0) &&
@@ -801,7 +803,7 @@ lddp_status lddp_plan(const lddp_desc* desc, lddp_plan_t* out) {
       // measured default (tools/gpu_hx5.sh, one B200): variant 2 (no lane ghosts, 64-row ring):
       // C4 2.00 -> 1.53 ms, C7 2.33 -> 1.55 ms
       const int hxv = env_int("LDDP_HX_VARIANT", 2);
-      if (hxv >= 0 && d.band_rows <= 0 && !(d.outputs & LDDP_OUT_TABLE) && d.cols > 0 && d.rows > 0 &&
+      if (hxv >= 0 && d.band_rows <= 0 && d.cols > 0 && d.rows > 0 &&
           d.cols % 4 == 0 && d.rows < (int64_t)1 << 30) {
         int q[3] = {0, 0, 0};
         FillParams dummy{};

@@ -99,7 +99,7 @@ struct Geo {
 }  // namespace hx
 
 // Per-lane state and the row loop of one warp.
-template <class F, int GH, int D>
+template <class F, int GH, int D, bool TB = false>
 struct HxLane {
   using T = typename F::T;
   using G = typename F::GridT;
@@ -112,6 +112,8 @@ struct HxLane {
   uint32_t pitchb;           // row pitch in bytes
   int hlast;                 // last table row (copies clamp to it)
   int e0;                    // first column of this lane
+  char* tptr;                // TB: &table[0][e0] (own in-table lanes), else nullptr
+  uint32_t tpitchb;          // TB: table row pitch in bytes
 
   __device__ __forceinline__ void issue(int rr, uint32_t dst) const {
     const int rc = min(rr, hlast);
@@ -170,14 +172,20 @@ struct HxLane {
         }
 #pragma unroll
         for (int j = 1 + t; j <= NX - 2 - t; ++j) x[j] = y[j];
+        if constexpr (TB) {   // TABLE: this row's own columns, one 16-byte store per lane
+          if (tptr != nullptr) {
+            char* d = tptr + (uint64_t)(uint32_t)(r + t) * tpitchb;
+            *reinterpret_cast<int4*>(d) = make_int4(x[GH], x[GH + 1], x[GH + 2], x[GH + 3]);
+          }
+        }
       }
     }
   }
 };
 
 // One band of HBI rows (FULL) or the last rows (r0 .. H-1, all already in the ring).
-template <class F, int GH, int D, int HBI, bool EDGE, bool FULL>
-__device__ __forceinline__ void hx_band(HxLane<F, GH, D>& st, const FillParams& p, int r0, int H) {
+template <class F, int GH, int D, bool TB, int HBI, bool EDGE, bool FULL>
+__device__ __forceinline__ void hx_band(HxLane<F, GH, D, TB>& st, const FillParams& p, int r0, int H) {
   constexpr int RB = hx::EXT * 4;
   if constexpr (FULL) {
     const int sl0 = r0 % D;
@@ -200,14 +208,14 @@ __device__ __forceinline__ void hx_band(HxLane<F, GH, D>& st, const FillParams& 
   }
 }
 
-template <class F, int NW, int HBI, int HBO, int D, int GH>
+template <class F, int NW, int HBI, int HBO, int D, int GH, bool TB>
 __global__ void __launch_bounds__(NW * 32, 1) prevrow_hx_kernel(const FillParams p) {
   using Geo = hx::Geo<NW, HBI, HBO>;
   static_assert(Geo::ok(), "hierarchical-exchange geometry");
   static_assert(D % HBI == 0 && HBI % GH == 0 && D > HBI + GH, "ring of whole bands");
   static_assert(!(F::kMask & NB_L), "prev-row category: f must not read L");
   using T = typename F::T;
-  using L = HxLane<F, GH, D>;
+  using L = HxLane<F, GH, D, TB>;
   constexpr int VP = hx::VP, EXT = hx::EXT, RB = EXT * 4;
   constexpr int CW = Geo::CW;
 
@@ -243,6 +251,8 @@ __global__ void __launch_bounds__(NW * 32, 1) prevrow_hx_kernel(const FillParams
   st.pitchb = (uint32_t)(p.grid_pitch * 4);
   st.hlast = H - 1;
   st.e0 = e0;
+  st.tptr = (TB && own && in) ? static_cast<char*>(p.table) + (int64_t)e0 * 4 : nullptr;
+  st.tpitchb = (uint32_t)(p.table_pitch * 4);
 
   // table-edge masks: every lane holding column 0 (v = 0) forces its UL, every lane holding column
   // W-1 (v = 3) its UR, to f's boundary values
@@ -298,11 +308,11 @@ __global__ void __launch_bounds__(NW * 32, 1) prevrow_hx_kernel(const FillParams
   for (int r0 = 0; r0 < H; r0 += HBI) {
     const long long tb0 = trc ? clock64() : 0;
     if (r0 + HBI <= H) {
-      if (edge) hx_band<F, GH, D, HBI, true, true>(st, p, r0, H);
-      else hx_band<F, GH, D, HBI, false, true>(st, p, r0, H);
+      if (edge) hx_band<F, GH, D, TB, HBI, true, true>(st, p, r0, H);
+      else hx_band<F, GH, D, TB, HBI, false, true>(st, p, r0, H);
     } else {
-      if (edge) hx_band<F, GH, D, HBI, true, false>(st, p, r0, H);
-      else hx_band<F, GH, D, HBI, false, false>(st, p, r0, H);
+      if (edge) hx_band<F, GH, D, TB, HBI, true, false>(st, p, r0, H);
+      else hx_band<F, GH, D, TB, HBI, false, false>(st, p, r0, H);
     }
     if (trc && r0 / HBI < 4096) p.trace[((r0 / HBI) * NW + w) * 2] = (uint64_t)(clock64() - tb0);
     if (r0 + HBI >= H) break;
@@ -409,8 +419,14 @@ template <class F, int NW, int HBI, int HBO, int D, int GH>
 static cudaError_t hx_launch(const FillParams& p, bool query, int* out, cudaStream_t s) {
   using Geo = hx::Geo<NW, HBI, HBO>;
   const size_t smem = 48 + (size_t)NW * D * hx::EXT * 4 + 2 * (size_t)NW * hx::EXT * 4 + 64;
-  auto k = prevrow_hx_kernel<F, NW, HBI, HBO, D, GH>;
-  cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  // TABLE fills: the TB instantiation (16-byte row stores; pitch and base checked by the caller)
+  auto k = p.table != nullptr ? prevrow_hx_kernel<F, NW, HBI, HBO, D, GH, true>
+                              : prevrow_hx_kernel<F, NW, HBI, HBO, D, GH, false>;
+  cudaError_t e = cudaFuncSetAttribute(prevrow_hx_kernel<F, NW, HBI, HBO, D, GH, true>,
+                                       cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(prevrow_hx_kernel<F, NW, HBI, HBO, D, GH, false>,
+                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   if (query) {   // out = {own columns per CTA, co-resident CTAs per SM, outer halo HBO}
     int occ = 0;

@@ -44,13 +44,17 @@ def test_minpath3_hx(hx_env, variant, shape):
     if -(-W // CTA_COLS[variant]) > 148:
         pytest.skip("more CTAs than SMs: the plan keeps prevrow_cb")
     c = inputs.gen_costs(31 * H + W, H, W)
-    ref = oracle.minpath3(c)
-    got = run_gpu("minpath3", "prev_row", grid=c, outputs=("score", "last_row"), reps=2)
+    tab = H * W <= 1 << 20
+    ref = oracle.minpath3(c, table=tab)
+    outs = ("score", "last_row", "table") if tab else ("score", "last_row")
+    got = run_gpu("minpath3", "prev_row", grid=c, outputs=outs, reps=2)
     info = json.loads(got["plan"])
     assert info["kernel"] == "prevrow_hx", info
     assert info["variant"] == variant
     np.testing.assert_array_equal(got["last_row"], ref.last_row)
     assert got["score"] == ref.score
+    if tab:
+        np.testing.assert_array_equal(got["table"], ref.table)
 
 
 @pytest.mark.parametrize("variant", VARIANTS)
@@ -59,15 +63,17 @@ def test_min2plus_diagmaxplus_hx(hx_env, variant, shape):
     hx_env(variant)
     H, W = shape
     init = inputs.gen_init(H + 5 * W, H, W, hi=10000)
-    ref = oracle.min2plus(init, 3)
-    got = run_gpu("min2plus", "prev_row", grid=init, param_c=3, outputs=("score", "last_row"))
+    ref = oracle.min2plus(init, 3, table=True)
+    got = run_gpu("min2plus", "prev_row", grid=init, param_c=3, outputs=("score", "last_row", "table"))
     assert json.loads(got["plan"])["kernel"] == "prevrow_hx"
     np.testing.assert_array_equal(got["last_row"], ref.last_row)
+    np.testing.assert_array_equal(got["table"], ref.table)
     assert got["score"] == ref.score
-    ref = oracle.diagmaxplus(init, 2)
-    got = run_gpu("diagmaxplus", "prev_row", grid=init, param_c=2, outputs=("last_row",))
+    ref = oracle.diagmaxplus(init, 2, table=True)
+    got = run_gpu("diagmaxplus", "prev_row", grid=init, param_c=2, outputs=("last_row", "table"))
     assert json.loads(got["plan"])["kernel"] == "prevrow_hx"
     np.testing.assert_array_equal(got["last_row"], ref.last_row)
+    np.testing.assert_array_equal(got["table"], ref.table)
 
 
 @pytest.mark.parametrize("variant", [0, 2])
@@ -83,13 +89,17 @@ def test_hx_pitched_grid(hx_env, variant):
 
 
 def test_hx_dispatch_rules(hx_env):
-    """TABLE outputs and an explicit band_rows keep the prevrow_cb kernel; HX_VARIANT=-1 too."""
+    """TABLE outputs run prevrow_hx too (16-byte row stores; a table pitch that is not a multiple
+    of 4 falls back to prevrow_cb at fill time); an explicit band_rows keeps prevrow_cb;
+    HX_VARIANT=-1 too."""
     hx_env(0)
     c = inputs.gen_costs(9, 300, 400)
     ref = oracle.minpath3(c, table=True)
     got = run_gpu("minpath3", "prev_row", grid=c, outputs=("score", "last_row", "table"))
-    assert json.loads(got["plan"])["kernel"] == "prevrow_cb"
+    assert json.loads(got["plan"])["kernel"] == "prevrow_hx"
     np.testing.assert_array_equal(got["table"], ref.table)
+    got = run_gpu("minpath3", "prev_row", grid=c, outputs=("score", "last_row", "table"), table_pad=3)
+    np.testing.assert_array_equal(got["table"], ref.table)   # pitch 403: the prevrow_cb fill
     got = run_gpu("minpath3", "prev_row", grid=c, outputs=("score", "last_row"), band_rows=32)
     assert json.loads(got["plan"])["kernel"] == "prevrow_cb"
     assert got["score"] == ref.score
