@@ -2,7 +2,7 @@
 measurement tool): LCS 8192² TABLE fills on the adiag staging-tile kernel and on the wavefront
 kernel, the traceback of that table, the claimed-task prev-row fallback (W % 4 != 0), the Vertical twin (transpose + prev-row),
 the mInverted-L twin (mirrored inverted-L), a batched FS fill (4 × 4096²) and a prev-row TABLE
-fill (prevrow_cb: the bench's prev-row lines run prevrow_hx).
+fill on prevrow_cb (LDDP_HX_VARIANT=-1; the bench's prev-row lines run prevrow_hx).
 
     ncu --set full -k regex:wavefront -c 1 python tools/prof_extra.py
 """
@@ -58,7 +58,9 @@ def main():
     del imgs, out
     gt = torch.from_numpy(inputs.gen_costs(3, n, n)).to(dev)
     tt = torch.zeros((n, n), dtype=torch.int32, device=dev)
+    os.environ["LDDP_HX_VARIANT"] = "-1"   # prevrow_cb (the multi-GPU / unaligned-TABLE kernel)
     p6 = lddp.Plan("minpath3", "prev_row", n, n, lddp.OUT_SCORE | lddp.OUT_TABLE)
+    del os.environ["LDDP_HX_VARIANT"]
     p6.fill(grid=gt, score=sc, table=tt)
     p6.check()
     torch.cuda.synchronize()
