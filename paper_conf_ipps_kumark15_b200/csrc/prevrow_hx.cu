@@ -1,28 +1,28 @@
 // prevrow_hx.cu -- previous-row-only ("Horizontal", t = i) category: hierarchical-exchange
-// column-block kernel, the default for SCORE / LAST_ROW fills (C4, C7) on one GPU [L180-L195],
-// Fig. 2(b).  prevrow_cb.cu remains the TABLE / multi-GPU / fallback path.
+// column-block kernel, the default prev-row kernel on one GPU (C4, C7; SCORE / LAST_ROW and
+// TABLE) [L180-L195], Fig. 2(b).  prevrow_cb.cu remains the multi-GPU / band_rows / unaligned-
+// TABLE path.
 //
 // Why a second column-block kernel.  prevrow_cb exchanges every warp's trapezoid halos through
 // L2 every HB = 32 rows; one store -> load visibility between SMs costs ~860 cycles
 // (tools/micro/l2rt.cu), the exchange is two-way, so every band pays C_band + ~1500 cycles on
-// the critical path: ~0.9 of C4's 2.0 ms.  Its row loop also re-forms the
-// 64-bit copy address and ring index per row (~31 issue slots per row) around a
-// SHFL -> VIMNMX3 -> IADD chain (~36 cycles of latency per row).  Here:
+// the critical path: ~0.9 of C4's 2.0 ms.  Here:
 //
 //  * Two exchange levels (Table II case-2 two-way halo [L265-L274], [L193-L195], applied
 //    hierarchically).  A CTA of NW warps (one per SM sub-partition) owns CW consecutive
 //    columns.  Warps of a CTA exchange their inner halos (HBI columns) through shared memory
 //    every HBI rows with one named barrier; only the CTA's two outer edges go through L2, every
 //    HBO rows, with HBO-column outer halos carried by the CTA's edge warps.  The L2 round trip
-//    is paid once per HBO rows instead of once per 32.
-//  * Lane ghosts (GH = 2): every lane keeps GH copies of each neighbour lane's edge columns and
-//    refreshes them by SHFL every GH rows, so the row chain is VIMNMX3 -> IADD with one SHFL
-//    per GH rows (garbage entering a lane window's edge advances one column per row -- the
-//    trapezoid argument one level down).  Costs of the row-0 ghost cells come by SHFL too.
+//    is paid once per HBO rows instead of once per 32.  Default HBI 16, HBO 96: C4 1.54 ms.
+//  * Optional lane ghosts (GH = 2, variant 0): every lane keeps GH copies of each neighbour
+//    lane's edge columns, refreshed by SHFL every GH rows (garbage entering a lane window's edge
+//    advances one column per row -- the trapezoid argument one level down); measured no faster
+//    than GH = 1 (the default), kept compiled.
 //  * A fully unrolled band: ring slots, LDS and LDGSTS destinations are immediates; one
 //    IMAD.WIDE forms each row's copy address; cp.async.wait once per GH rows.
 //  * Table edges: column 0's UL and column W-1's UR are forced to f's boundary value with one
 //    LOP3 each in the (warp-uniform) EDGE body only, in every lane that holds those columns.
+//  * TABLE (TB): every own in-table lane stores its 4 new values per row with one 16-byte store.
 //
 // Geometry: lane l of warp w holds the VP = 4 columns [s_w + 4l, s_w + 4l + 4) of the warp's
 // window [s_w, s_w + 128); hl(w) = HBO for w = 0 else HBI columns of left halo, hr(w) likewise
