@@ -140,6 +140,10 @@ const AdGeom kAdGeoms[] = {
 LDDP_AD_TABLE_ROWS
 };
 
+// prev-row multi-GPU: edge pairs per slot and side in the comm window (>= HB of prevrow_cb and
+// HBO of prevrow_hx)
+constexpr int kHaloSide = 96;
+
 bool ad_has_table(int func) {
   for (const auto& g : kAdGeoms)
     if (g.func == func && g.TB) return true;
@@ -249,7 +253,7 @@ struct lddp_comm_s {
   int nranks, rank, device;
   void* window;          // this rank's window (device memory of this rank)
   size_t win_bytes;
-  size_t off_flag, off_val, off_halo;   // off_halo: prev-row edges [from left 8 x 64][from right 8 x 64]
+  size_t off_flag, off_val, off_halo;   // off_halo: prev-row edges [from left 8 x kHaloSide][from right ...]
   int64_t nstrips, rows;
   void* next;            // rank+1's window (IPC-opened or in-process), NULL on the last rank
   void* prev;            // rank-1's window, NULL on rank 0
@@ -1063,7 +1067,13 @@ lddp_status lddp_multi_partition(int64_t cols, int32_t nranks, int32_t rank, int
 // The share of rank `rank` of `nranks` in a multi-GPU fill of this plan: columns [lo, hi) for
 // column strips (anti-diagonal: near-equal; prev-row: whole column blocks of the column-block
 // kernel), diagonals d = j - i in [lo, hi) for inverted-L diagonal shares (~1/P of the cells).
-static void plan_share(lddp_plan_t pl, int32_t nranks, int32_t rank, int64_t* lo, int64_t* hi) {
+static // lddp_fill_multi runs a prev-row plan on prevrow_hx when the plan has it and every rank gets at
+// least one whole CTA strip (the partition is then CTA-aligned); prevrow_cb otherwise
+bool prev_multi_hx(const lddp_plan_s* pl, int nranks) {
+  return pl->hx_variant >= 0 && (pl->desc.cols + pl->hx_cw - 1) / pl->hx_cw >= nranks;
+}
+
+void plan_share(lddp_plan_t pl, int32_t nranks, int32_t rank, int64_t* lo, int64_t* hi) {
   const lddp_desc& d = pl->desc;
   const int64_t H = d.rows, W = d.cols;
   if (pl->kind == 2) {
@@ -1086,8 +1096,8 @@ static void plan_share(lddp_plan_t pl, int32_t nranks, int32_t rank, int64_t* lo
     const int64_t B = std::max(d.batch, 1);   // batched FS: images
     *lo = (int64_t)rank * B / nranks;
     *hi = (int64_t)(rank + 1) * B / nranks;
-  } else if (pl->kind == 1 && pl->cb_variant >= 0) {
-    const int64_t BW = pl->cb_bw;
+  } else if (pl->kind == 1 && (pl->cb_variant >= 0 || prev_multi_hx(pl, nranks))) {
+    const int64_t BW = prev_multi_hx(pl, nranks) ? pl->hx_cw : pl->cb_bw;
     const int64_t NB = (W + BW - 1) / BW;
     const int64_t b0 = (int64_t)rank * NB / nranks, b1 = (int64_t)(rank + 1) * NB / nranks;
     *lo = std::min<int64_t>(b0 * BW, W);
@@ -1129,7 +1139,7 @@ lddp_status lddp_comm_create(lddp_plan_t pl, int32_t nranks, int32_t rank, lddp_
   c->off_flag = align_up((size_t)2 * c->nstrips * 8, 256);
   c->off_val = c->off_flag + align_up((size_t)2 * c->nstrips * 8, 256);
   c->off_halo = align_up(c->off_val + (size_t)2 * (c->rows + 1) * 4, 256);
-  c->win_bytes = c->off_halo + (size_t)2 * 8 * 64 * 8;
+  c->win_bytes = c->off_halo + (size_t)2 * 8 * kHaloSide * 8;
   cudaError_t e = cudaMalloc(&c->window, c->win_bytes);
   if (e == cudaSuccess) e = cudaMemset(c->window, 0, c->win_bytes);
   if (e != cudaSuccess) {
@@ -1330,14 +1340,24 @@ lddp_status lddp_fill_multi(lddp_plan_t pl, const lddp_inputs* in, const lddp_ou
       uint64_t* own = reinterpret_cast<uint64_t*>(static_cast<char*>(c->window) + c->off_halo);
       if (c->rank > 0) {
         p.halo_in_l = own;                                                                   // from left
-        p.halo_out_l = reinterpret_cast<uint64_t*>(static_cast<char*>(c->prev) + c->off_halo) + 8 * 64;   // its "from right"
+        p.halo_out_l = reinterpret_cast<uint64_t*>(static_cast<char*>(c->prev) + c->off_halo) + 8 * kHaloSide;   // its "from right"
       }
       if (c->rank < c->nranks - 1) {
-        p.halo_in_r = own + 8 * 64;                                                          // from right
+        p.halo_in_r = own + 8 * kHaloSide;                                                   // from right
         p.halo_out_r = reinterpret_cast<uint64_t*>(static_cast<char*>(c->next) + c->off_halo);            // its "from left"
       }
-      int dummy2[2];
-      cudaError_t e = lddp::launch_prevrow_cb(d.func, pl->cb_variant, p, pl->cb_nw, false, dummy2, s);
+      cudaError_t e;
+      if (prev_multi_hx(pl, c->nranks)) {
+        // hierarchical-exchange kernel: CTA-aligned strips, the strip's outer CTA edges through
+        // the windows every HBO rows (TABLE: 16-byte row stores)
+        if (p.table != nullptr && ((p.table_pitch % 4) || (reinterpret_cast<uintptr_t>(p.table) & 15)))
+          return fail(LDDP_ERR_UNSUPPORTED, "multi-GPU prev-row TABLE: 16-byte aligned table, pitch %% 4 == 0");
+        int dummy3[3];
+        e = lddp::launch_prevrow_hx(d.func, pl->hx_variant, p, false, dummy3, s);
+      } else {
+        int dummy2[2];
+        e = lddp::launch_prevrow_cb(d.func, pl->cb_variant, p, pl->cb_nw, false, dummy2, s);
+      }
       if (e != cudaSuccess) return cuda_fail(e, "kernel launch");
       return LDDP_OK;
     }

@@ -69,6 +69,13 @@ __device__ __forceinline__ void st_pair2(uint64_t* p, uint64_t a, uint64_t b) {
 __device__ __forceinline__ void ld_pair2(const uint64_t* p, uint64_t& a, uint64_t& b) {
   asm volatile("ld.relaxed.gpu.global.v2.u64 {%0, %1}, [%2];" : "=l"(a), "=l"(b) : "l"(p) : "memory");
 }
+// system scope: edge pairs exchanged with the neighbour GPUs' comm windows (lddp_fill_multi)
+__device__ __forceinline__ void st_pair2_sys(uint64_t* p, uint64_t a, uint64_t b) {
+  asm volatile("st.relaxed.sys.global.v2.u64 [%0], {%1, %2};" ::"l"(p), "l"(a), "l"(b) : "memory");
+}
+__device__ __forceinline__ void ld_pair2_sys(const uint64_t* p, uint64_t& a, uint64_t& b) {
+  asm volatile("ld.relaxed.sys.global.v2.u64 {%0, %1}, [%2];" : "=l"(a), "=l"(b) : "l"(p) : "memory");
+}
 __device__ __forceinline__ uint32_t opq(uint32_t x) {
   asm volatile("mov.b32 %0, %0;" : "+r"(x));
   return x;
@@ -245,9 +252,14 @@ __global__ void __launch_bounds__(NW * 32, 1) prevrow_hx_kernel(const FillParams
   st.ring0 = sbase + 16 + (uint32_t)(w * D * RB + lane * 16);
   const uint32_t xs0 = sbase + 32 + (uint32_t)(NW * D * RB);
   const int xidx = e0 - (A - HBO);       // index in the CTA's extended window
-  const bool in = e0 >= 0 && e0 < W;     // W % 4 == 0: a lane's 4 columns are all in or all out
-  st.gsz = hx::opq(in ? 16u : 0u);
-  st.gsrc = static_cast<const char*>(p.grid) + (in ? (int64_t)e0 * 4 : 0);
+  // local columns: [0, W) this rank's strip (outputs); [clo, chi) the whole table (costs: a
+  // multi-GPU rank's halos read its neighbours' columns of the grid).  W % 4 == 0 and the strip
+  // starts on a multiple of 4: a lane's 4 columns are all in or all out.
+  const int clo = -p.col0, chi = p.cols_total - p.col0;
+  const bool in = e0 >= 0 && e0 < W;
+  const bool gin = e0 >= clo && e0 < chi;
+  st.gsz = hx::opq(gin ? 16u : 0u);
+  st.gsrc = static_cast<const char*>(p.grid) + (gin ? (int64_t)e0 * 4 : 0);
   st.pitchb = (uint32_t)(p.grid_pitch * 4);
   st.hlast = H - 1;
   st.e0 = e0;
@@ -261,16 +273,16 @@ __global__ void __launch_bounds__(NW * 32, 1) prevrow_hx_kernel(const FillParams
     uint32_t lbits, rbits;
     memcpy(&lbits, &lb, 4);
     memcpy(&rbits, &rb, 4);
-    st.lA = hx::opq(e0 == 0 ? 0u : ~0u);
-    st.lO = hx::opq(e0 == 0 ? lbits : 0u);
-    st.rA = hx::opq(e0 == W - VP ? 0u : ~0u);
-    st.rO = hx::opq(e0 == W - VP ? rbits : 0u);
+    st.lA = hx::opq(e0 == clo ? 0u : ~0u);
+    st.lO = hx::opq(e0 == clo ? lbits : 0u);
+    st.rA = hx::opq(e0 == chi - VP ? 0u : ~0u);
+    st.rO = hx::opq(e0 == chi - VP ? rbits : 0u);
   }
-  const bool edge = __any_sync(0xffffffffu, e0 == 0 || e0 == W - VP);
+  const bool edge = __any_sync(0xffffffffu, e0 == clo || e0 == chi - VP);
 
   // row -1 (virtual): f's top initialisation (out-of-table columns: garbage, never read)
 #pragma unroll
-  for (int v = 0; v < VP; ++v) st.x[GH + v] = F::top(p, e0 + v);
+  for (int v = 0; v < VP; ++v) st.x[GH + v] = F::top(p, p.col0 + e0 + v);
 
   // prologue: rows 0 .. D-2 into slots 0 .. D-2
 #pragma unroll 1
@@ -278,18 +290,31 @@ __global__ void __launch_bounds__(NW * 32, 1) prevrow_hx_kernel(const FillParams
 
   // outer-edge pairs in global memory: [CTA][4 slots][2 sides][HBO] (value, tag)
   uint64_t* edges = reinterpret_cast<uint64_t*>(p.bnd);
-  const uint32_t tag0 = (uint32_t)(p.epoch & 0x7FFu) << 20;
+  // multi-GPU (lddp_fill_multi): CTA 0's left and the last CTA's right outer edges go to / come
+  // from the neighbour ranks' comm windows ([8 slots: fill parity x outer band mod 4][HBO] pairs
+  // per side, system scope); the strip partition is CTA-aligned, so the rank's strip edges are
+  // CTA edges.  Tags carry the rank-consistent fill count (bit 31 set).
+  const bool xrank = p.halo_in_l != nullptr || p.halo_in_r != nullptr;
+  const uint32_t tag0 = xrank ? (0x80000000u | (uint32_t)(p.wepoch & 0x7FFu) << 20) : (uint32_t)(p.epoch & 0x7FFu) << 20;
   const bool pub_l = own && e0 >= A && e0 < A + HBO;               // CTA c-1 reads these
   const bool pub_r = own && e0 >= A + CW - HBO && e0 < A + CW;     // CTA c+1 reads these
-  const bool get_l = w == 0 && lhalo && c > 0;
-  const bool get_r = w == NW - 1 && rhalo && c + 1 < nc;
+  const bool xin = (w == 0 && lhalo && c == 0 && p.halo_in_l != nullptr) ||
+                   (w == NW - 1 && rhalo && c + 1 == nc && p.halo_in_r != nullptr);
+  const bool get_l = w == 0 && lhalo && (c > 0 || p.halo_in_l != nullptr);
+  const bool get_r = w == NW - 1 && rhalo && (c + 1 < nc || p.halo_in_r != nullptr);
+  uint64_t* const xout = (pub_l && c == 0 && p.halo_out_l != nullptr) ? p.halo_out_l + (e0 - A)
+                         : ((pub_r && c + 1 == nc && p.halo_out_r != nullptr) ? p.halo_out_r + (e0 - (A + CW - HBO))
+                                                                               : nullptr);
   const bool pub = pub_l || pub_r, get = get_l || get_r;
   const bool ihalo = !own && !((w == 0 && lhalo) || (w == NW - 1 && rhalo));   // inner halo lane
   // this lane's pair addresses in slot 0 (slot s adds s * 2 * HBO): own edge columns it publishes,
   // neighbour columns it polls
   uint64_t* const pubp = edges + ((size_t)c * 8 + (pub_l ? 0 : 1)) * HBO + (pub_l ? e0 - A : e0 - (A + CW - HBO));
-  const uint64_t* const getp = get_l ? edges + ((size_t)(c - 1) * 8 + 1) * HBO + (e0 - (A - HBO))
-                                     : edges + ((size_t)(c + 1) * 8 + 0) * HBO + (e0 - (A + CW));
+  const uint64_t* const getp =
+      xin ? (get_l ? p.halo_in_l + (e0 - (A - HBO)) : p.halo_in_r + (e0 - (A + CW)))
+          : (get_l ? edges + ((size_t)(c - 1) * 8 + 1) * HBO + (e0 - (A - HBO))
+                   : edges + ((size_t)(c + 1) * 8 + 0) * HBO + (e0 - (A + CW)));
+  const size_t xpar_slot = (size_t)(p.wepoch & 1) * 4;   // window slot base of this fill
   const uint32_t xsa = xs0 + (uint32_t)(xidx * 4);
   uint32_t xpar = 0;
   int kin = 0, ob = 0;   // inner band within the outer band, outer band
@@ -329,6 +354,11 @@ __global__ void __launch_bounds__(NW * 32, 1) prevrow_hx_kernel(const FillParams
       const uint64_t th = (uint64_t)tag << 32;
       hx::st_pair2(d, th | (uint32_t)st.x[GH], th | (uint32_t)st.x[GH + 1]);
       hx::st_pair2(d + 2, th | (uint32_t)st.x[GH + 2], th | (uint32_t)st.x[GH + 3]);
+      if (xout != nullptr) {   // the strip's outer edge -> the neighbour rank's window
+        uint64_t* x = xout + (xpar_slot + (ob & 3)) * HBO;
+        hx::st_pair2_sys(x, th | (uint32_t)st.x[GH], th | (uint32_t)st.x[GH + 1]);
+        hx::st_pair2_sys(x + 2, th | (uint32_t)st.x[GH + 2], th | (uint32_t)st.x[GH + 3]);
+      }
     }
     if (!dbg_no_inner) {
       hx::bar_named<NW * 32>();
@@ -338,13 +368,18 @@ __global__ void __launch_bounds__(NW * 32, 1) prevrow_hx_kernel(const FillParams
       }
     }
     if (outer && (w == 0 || w == NW - 1) && !dbg_no_outer) {
-      const uint64_t* s = getp + (size_t)(ob & 3) * 2 * HBO;
+      const uint64_t* s = getp + (xin ? (xpar_slot + (ob & 3)) * HBO : (size_t)(ob & 3) * 2 * HBO);
       const bool need = get && !aborted;
       uint64_t pr[VP];
       bool ok = true;
       if (need) {
-        hx::ld_pair2(s, pr[0], pr[1]);
-        hx::ld_pair2(s + 2, pr[2], pr[3]);
+        if (xin) {
+          hx::ld_pair2_sys(s, pr[0], pr[1]);
+          hx::ld_pair2_sys(s + 2, pr[2], pr[3]);
+        } else {
+          hx::ld_pair2(s, pr[0], pr[1]);
+          hx::ld_pair2(s + 2, pr[2], pr[3]);
+        }
 #pragma unroll
         for (int v = 0; v < VP; ++v) ok = ok && ((uint32_t)(pr[v] >> 32) == tag);
       }
@@ -353,8 +388,13 @@ __global__ void __launch_bounds__(NW * 32, 1) prevrow_hx_kernel(const FillParams
         int spins = 0;
         while (true) {
           if (!ok) {
-            hx::ld_pair2(s, pr[0], pr[1]);
-            hx::ld_pair2(s + 2, pr[2], pr[3]);
+            if (xin) {
+              hx::ld_pair2_sys(s, pr[0], pr[1]);
+              hx::ld_pair2_sys(s + 2, pr[2], pr[3]);
+            } else {
+              hx::ld_pair2(s, pr[0], pr[1]);
+              hx::ld_pair2(s + 2, pr[2], pr[3]);
+            }
             ok = true;
 #pragma unroll
             for (int v = 0; v < VP; ++v) ok = ok && ((uint32_t)(pr[v] >> 32) == tag);

@@ -9,6 +9,7 @@
   fill's column.  Each result must equal the oracle.
 * Cross-process: 2-3 processes on the same GPU exchange CUDA IPC window handles over a gloo
   process group (lddp_comm_handle / lddp_comm_connect), the path bench.py takes across GPUs."""
+import json
 import os
 import socket
 import time
@@ -232,9 +233,10 @@ def test_inverted_l_diagonal_shares(func, cat, P, shape):
 @pytest.mark.parametrize("func", ["minpath3", "min2plus"])
 @pytest.mark.parametrize("P", [2, 3, 4])
 @pytest.mark.parametrize("shape", [(300, 1024), (1000, 2048), (517, 1540), (64, 4096)])
-def test_prev_row_two_way_halos(func, P, shape):
+@pytest.mark.parametrize("kernel", ["prevrow_hx", "prevrow_cb"])
+def test_prev_row_two_way_halos(func, P, shape, kernel, monkeypatch):
     """Previous-row category across P ranks (loopback: all ranks on this GPU, each with its own
-    window, workspace and stream): block-aligned column strips; every band the strips' outer
+    window, workspace and stream), on both prev-row kernels: CTA- / block-aligned column strips; every band the strips' outer
     blocks exchange their HB-column edges with the neighbour ranks both ways (Table II case 2,
     [L193-L195], [L265-L274]).  Several fills with different grids, enqueued rank by rank.  The
     score is per rank (the minimum of its columns); its minimum over ranks is the oracle's."""
@@ -243,7 +245,10 @@ def test_prev_row_two_way_halos(func, P, shape):
     from paper_conf_ipps_kumark15_b200 import lddp
     H, W = shape
     dev = torch.device("cuda:0")
+    if kernel == "prevrow_cb":   # the hierarchical-exchange kernel is the default when it fits
+        monkeypatch.setenv("LDDP_HX_VARIANT", "-1")
     plan = lddp.Plan(func, "prev_row", H, W, lddp.OUT_SCORE | lddp.OUT_LAST_ROW | lddp.OUT_TABLE)
+    assert json.loads(plan.info)["kernel"] == kernel
     comms = [lddp.lddp_comm_create(plan.handle, P, r) for r in range(P)]
     for r in range(P):
         lddp.lddp_comm_connect_local(comms[r], comms[r + 1] if r + 1 < P else None, comms[r - 1] if r > 0 else None)
