@@ -143,9 +143,10 @@ typedef struct {
     int32_t band_rows;       /* tuning, prev-row category: trapezoid band height HB (rows between
                                 two halo exchanges of the column-block kernel prevrow_cb): 16,
                                 32, 48 or 64 (else LDDP_ERR_UNSUPPORTED); 0 = auto (SCORE /
-                                LAST_ROW / TABLE fills on one GPU: the hierarchical-exchange
-                                kernel, inner halos every 16 rows, CTA-edge halos every 96;
-                                lddp_fill_multi and TABLE pitches that are not multiples of 4:
+                                LAST_ROW / TABLE fills, also lddp_fill_multi: the hierarchical-
+                                exchange kernel, inner halos every 16 rows, CTA-edge halos
+                                every 96; TABLE pitches that are not multiples of 4, and
+                                multi-GPU plans too narrow for one CTA strip per rank:
                                 prevrow_cb with HB = 32)                                        */
     int32_t grid_ctas;       /* tuning: persistent grid size, 0 = auto (SMs x occupancy)        */
     int32_t batch;           /* FS_DITHER only: number of independent images stacked along the
