@@ -817,11 +817,13 @@ lddp_status lddp_plan(const lddp_desc* desc, lddp_plan_t* out) {
             pl->hx_variant = hxv;
             pl->hx_cw = q[0];
             pl->hx_ctas = (int)ctas;
-            // workspace: per-CTA row minima + outer edge pairs [CTA][4 slots][2 sides][HBO] x 8 B
+            // workspace: per-CTA row minima + outer edge pairs [CTA][4 slots][2 sides][HBO] x 8 B,
+            // or for one-way f's (no UR) [CTA][one slot per outer band][HBO]
             const size_t prog = align_up(64 + (size_t)ctas * 4, 256);
+            const int64_t nob = (d.rows + q[2] - 1) / q[2];
             pl->off_prog = 64;
             pl->off_bnd = std::max(pl->off_bnd, prog);
-            pl->ws_bytes = std::max(pl->ws_bytes, pl->off_bnd + (size_t)ctas * 4 * 2 * q[2] * 8);
+            pl->ws_bytes = std::max(pl->ws_bytes, pl->off_bnd + (size_t)ctas * std::max<int64_t>(8, nob) * q[2] * 8);
           }
         } else {
           cudaGetLastError();
@@ -1067,13 +1069,13 @@ lddp_status lddp_multi_partition(int64_t cols, int32_t nranks, int32_t rank, int
 // The share of rank `rank` of `nranks` in a multi-GPU fill of this plan: columns [lo, hi) for
 // column strips (anti-diagonal: near-equal; prev-row: whole column blocks of the column-block
 // kernel), diagonals d = j - i in [lo, hi) for inverted-L diagonal shares (~1/P of the cells).
-static // lddp_fill_multi runs a prev-row plan on prevrow_hx when the plan has it and every rank gets at
+// lddp_fill_multi runs a prev-row plan on prevrow_hx when the plan has it and every rank gets at
 // least one whole CTA strip (the partition is then CTA-aligned); prevrow_cb otherwise
-bool prev_multi_hx(const lddp_plan_s* pl, int nranks) {
+static bool prev_multi_hx(const lddp_plan_s* pl, int nranks) {
   return pl->hx_variant >= 0 && (pl->desc.cols + pl->hx_cw - 1) / pl->hx_cw >= nranks;
 }
 
-void plan_share(lddp_plan_t pl, int32_t nranks, int32_t rank, int64_t* lo, int64_t* hi) {
+static void plan_share(lddp_plan_t pl, int32_t nranks, int32_t rank, int64_t* lo, int64_t* hi) {
   const lddp_desc& d = pl->desc;
   const int64_t H = d.rows, W = d.cols;
   if (pl->kind == 2) {

@@ -215,7 +215,7 @@ __device__ __forceinline__ void hx_band(HxLane<F, GH, D, TB>& st, const FillPara
   }
 }
 
-template <class F, int NW, int HBI, int HBO, int D, int GH, bool TB>
+template <class F, int NW, int HBI, int HBO, int D, int GH, bool TB, bool XR>
 __global__ void __launch_bounds__(NW * 32, 1) prevrow_hx_kernel(const FillParams p) {
   using Geo = hx::Geo<NW, HBI, HBO>;
   static_assert(Geo::ok(), "hierarchical-exchange geometry");
@@ -255,7 +255,8 @@ __global__ void __launch_bounds__(NW * 32, 1) prevrow_hx_kernel(const FillParams
   // local columns: [0, W) this rank's strip (outputs); [clo, chi) the whole table (costs: a
   // multi-GPU rank's halos read its neighbours' columns of the grid).  W % 4 == 0 and the strip
   // starts on a multiple of 4: a lane's 4 columns are all in or all out.
-  const int clo = -p.col0, chi = p.cols_total - p.col0;
+  // (XR: a multi-GPU rank's fill; the single-GPU instantiation keeps the window code out)
+  const int clo = XR ? -p.col0 : 0, chi = XR ? p.cols_total - p.col0 : W;
   const bool in = e0 >= 0 && e0 < W;
   const bool gin = e0 >= clo && e0 < chi;
   st.gsz = hx::opq(gin ? 16u : 0u);
@@ -294,26 +295,39 @@ __global__ void __launch_bounds__(NW * 32, 1) prevrow_hx_kernel(const FillParams
   // from the neighbour ranks' comm windows ([8 slots: fill parity x outer band mod 4][HBO] pairs
   // per side, system scope); the strip partition is CTA-aligned, so the rank's strip edges are
   // CTA edges.  Tags carry the rank-consistent fill count (bit 31 set).
-  const bool xrank = p.halo_in_l != nullptr || p.halo_in_r != nullptr;
+  constexpr bool xrank = XR;
   const uint32_t tag0 = xrank ? (0x80000000u | (uint32_t)(p.wepoch & 0x7FFu) << 20) : (uint32_t)(p.epoch & 0x7FFu) << 20;
-  const bool pub_l = own && e0 >= A && e0 < A + HBO;               // CTA c-1 reads these
+  // One-way f's (contributing set without UR: MIN2_PLUS, DIAG_MAXPLUS -- Table II case 1, one-way
+  // transfer [L265-L274]): own columns depend only on columns to their left, so a CTA waits for
+  // its left neighbour's edge and never for its right one -- the CTAs form a pipeline instead of
+  // a lock-step chain.  With no back-pressure a producer may run any number of outer bands
+  // ahead, so (one GPU) every outer band has its own slot: edges[CTA][NOB][HBO], never reused
+  // within a fill (the tags tell fills apart).
+  constexpr bool kOneWayF = !(F::kMask & NB_UR);
+  const bool oneway = kOneWayF && !xrank;
+  const int NOB = (H + HBO - 1) / HBO;
+  const bool pub_l = own && e0 >= A && e0 < A + HBO && !oneway;    // CTA c-1 reads these
   const bool pub_r = own && e0 >= A + CW - HBO && e0 < A + CW;     // CTA c+1 reads these
-  const bool xin = (w == 0 && lhalo && c == 0 && p.halo_in_l != nullptr) ||
-                   (w == NW - 1 && rhalo && c + 1 == nc && p.halo_in_r != nullptr);
-  const bool get_l = w == 0 && lhalo && (c > 0 || p.halo_in_l != nullptr);
-  const bool get_r = w == NW - 1 && rhalo && (c + 1 < nc || p.halo_in_r != nullptr);
-  uint64_t* const xout = (pub_l && c == 0 && p.halo_out_l != nullptr) ? p.halo_out_l + (e0 - A)
+  const bool xin = XR && ((w == 0 && lhalo && c == 0 && p.halo_in_l != nullptr) ||
+                          (w == NW - 1 && rhalo && c + 1 == nc && p.halo_in_r != nullptr));
+  const bool get_l = w == 0 && lhalo && (c > 0 || (XR && p.halo_in_l != nullptr));
+  const bool get_r = w == NW - 1 && rhalo && (c + 1 < nc || (XR && p.halo_in_r != nullptr)) && !oneway;
+  uint64_t* const xout = !XR ? nullptr
+                         : (pub_l && c == 0 && p.halo_out_l != nullptr) ? p.halo_out_l + (e0 - A)
                          : ((pub_r && c + 1 == nc && p.halo_out_r != nullptr) ? p.halo_out_r + (e0 - (A + CW - HBO))
                                                                                : nullptr);
   const bool pub = pub_l || pub_r, get = get_l || get_r;
   const bool ihalo = !own && !((w == 0 && lhalo) || (w == NW - 1 && rhalo));   // inner halo lane
   // this lane's pair addresses in slot 0 (slot s adds s * 2 * HBO): own edge columns it publishes,
   // neighbour columns it polls
-  uint64_t* const pubp = edges + ((size_t)c * 8 + (pub_l ? 0 : 1)) * HBO + (pub_l ? e0 - A : e0 - (A + CW - HBO));
+  uint64_t* const pubp =
+      oneway ? edges + (size_t)c * NOB * HBO + (e0 - (A + CW - HBO))
+             : edges + ((size_t)c * 8 + (pub_l ? 0 : 1)) * HBO + (pub_l ? e0 - A : e0 - (A + CW - HBO));
   const uint64_t* const getp =
       xin ? (get_l ? p.halo_in_l + (e0 - (A - HBO)) : p.halo_in_r + (e0 - (A + CW)))
-          : (get_l ? edges + ((size_t)(c - 1) * 8 + 1) * HBO + (e0 - (A - HBO))
-                   : edges + ((size_t)(c + 1) * 8 + 0) * HBO + (e0 - (A + CW)));
+          : (oneway ? edges + (size_t)(c - 1) * NOB * HBO + (e0 - (A - HBO))
+                    : (get_l ? edges + ((size_t)(c - 1) * 8 + 1) * HBO + (e0 - (A - HBO))
+                             : edges + ((size_t)(c + 1) * 8 + 0) * HBO + (e0 - (A + CW))));
   const size_t xpar_slot = (size_t)(p.wepoch & 1) * 4;   // window slot base of this fill
   const uint32_t xsa = xs0 + (uint32_t)(xidx * 4);
   uint32_t xpar = 0;
@@ -349,12 +363,13 @@ __global__ void __launch_bounds__(NW * 32, 1) prevrow_hx_kernel(const FillParams
     const bool outer = kin == HBO / HBI - 1;   // an outer band (HBO rows) ends here
     kin = outer ? 0 : kin + 1;
     const uint32_t tag = tag0 | (((uint32_t)ob + 1u) & 0xFFFFFu);
+    const size_t soff = oneway ? (size_t)ob * HBO : (size_t)(ob & 3) * 2 * HBO;   // this band's slot
     if (outer && pub) {
-      uint64_t* d = pubp + (size_t)(ob & 3) * 2 * HBO;
+      uint64_t* d = pubp + soff;
       const uint64_t th = (uint64_t)tag << 32;
       hx::st_pair2(d, th | (uint32_t)st.x[GH], th | (uint32_t)st.x[GH + 1]);
       hx::st_pair2(d + 2, th | (uint32_t)st.x[GH + 2], th | (uint32_t)st.x[GH + 3]);
-      if (xout != nullptr) {   // the strip's outer edge -> the neighbour rank's window
+      if (XR && xout != nullptr) {   // the strip's outer edge -> the neighbour rank's window
         uint64_t* x = xout + (xpar_slot + (ob & 3)) * HBO;
         hx::st_pair2_sys(x, th | (uint32_t)st.x[GH], th | (uint32_t)st.x[GH + 1]);
         hx::st_pair2_sys(x + 2, th | (uint32_t)st.x[GH + 2], th | (uint32_t)st.x[GH + 3]);
@@ -368,12 +383,12 @@ __global__ void __launch_bounds__(NW * 32, 1) prevrow_hx_kernel(const FillParams
       }
     }
     if (outer && (w == 0 || w == NW - 1) && !dbg_no_outer) {
-      const uint64_t* s = getp + (xin ? (xpar_slot + (ob & 3)) * HBO : (size_t)(ob & 3) * 2 * HBO);
+      const uint64_t* s = getp + (xin ? (xpar_slot + (ob & 3)) * HBO : soff);
       const bool need = get && !aborted;
       uint64_t pr[VP];
       bool ok = true;
       if (need) {
-        if (xin) {
+        if (XR && xin) {
           hx::ld_pair2_sys(s, pr[0], pr[1]);
           hx::ld_pair2_sys(s + 2, pr[2], pr[3]);
         } else {
@@ -388,7 +403,7 @@ __global__ void __launch_bounds__(NW * 32, 1) prevrow_hx_kernel(const FillParams
         int spins = 0;
         while (true) {
           if (!ok) {
-            if (xin) {
+            if (XR && xin) {
               hx::ld_pair2_sys(s, pr[0], pr[1]);
               hx::ld_pair2_sys(s + 2, pr[2], pr[3]);
             } else {
@@ -459,14 +474,17 @@ template <class F, int NW, int HBI, int HBO, int D, int GH>
 static cudaError_t hx_launch(const FillParams& p, bool query, int* out, cudaStream_t s) {
   using Geo = hx::Geo<NW, HBI, HBO>;
   const size_t smem = 48 + (size_t)NW * D * hx::EXT * 4 + 2 * (size_t)NW * hx::EXT * 4 + 64;
-  // TABLE fills: the TB instantiation (16-byte row stores; pitch and base checked by the caller)
-  auto k = p.table != nullptr ? prevrow_hx_kernel<F, NW, HBI, HBO, D, GH, true>
-                              : prevrow_hx_kernel<F, NW, HBI, HBO, D, GH, false>;
-  cudaError_t e = cudaFuncSetAttribute(prevrow_hx_kernel<F, NW, HBI, HBO, D, GH, true>,
-                                       cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  if (e == cudaSuccess)
-    e = cudaFuncSetAttribute(prevrow_hx_kernel<F, NW, HBI, HBO, D, GH, false>,
-                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  // TABLE fills: the TB instantiation (16-byte row stores; pitch and base checked by the caller);
+  // multi-GPU rank fills: the XR instantiation (comm-window edges)
+  const bool xr = p.halo_in_l != nullptr || p.halo_in_r != nullptr;
+  decltype(&prevrow_hx_kernel<F, NW, HBI, HBO, D, GH, false, false>) ks[2][2] = {
+      {prevrow_hx_kernel<F, NW, HBI, HBO, D, GH, false, false>, prevrow_hx_kernel<F, NW, HBI, HBO, D, GH, false, true>},
+      {prevrow_hx_kernel<F, NW, HBI, HBO, D, GH, true, false>, prevrow_hx_kernel<F, NW, HBI, HBO, D, GH, true, true>}};
+  auto k = ks[p.table != nullptr][xr];
+  cudaError_t e = cudaSuccess;
+  for (int a = 0; a < 2 && e == cudaSuccess; ++a)
+    for (int b = 0; b < 2 && e == cudaSuccess; ++b)
+      e = cudaFuncSetAttribute(ks[a][b], cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   if (query) {   // out = {own columns per CTA, co-resident CTAs per SM, outer halo HBO}
     int occ = 0;
