@@ -1,6 +1,6 @@
 export LDDP_TIMEOUT_MS=5000
 timeout 600 python -m pytest tests/test_gpu_prevrow_hx.py -x -q > gpurun_out/hx_t.log 2>&1; tail -15 gpurun_out/hx_t.log
-timeout 300 python tools/quick_time.py C4 C7 --env LDDP_HX_VARIANT=-1,0,1,2,3,4,5 --reps 5 > gpurun_out/hx_q.log 2>&1; grep -v '^#' gpurun_out/hx_q.log | python -c "
+timeout 300 python tools/quick_time.py C4 C7 --env LDDP_HX_VARIANT=-1,0,2,6,8 --reps 5 > gpurun_out/hx_q.log 2>&1; grep -v '^#' gpurun_out/hx_q.log | python -c "
 import sys,json
 for l in sys.stdin:
     try: d=json.loads(l)
